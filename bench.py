@@ -1,0 +1,423 @@
+#!/usr/bin/env python
+"""bench.py -- device-timed matches/s of the batched message-matching hot path.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--levels mpi,ordered,unordered]
+
+One step = one mm_match_batch over one batch of synthetic input (posted
+receives + arrived messages already resident in HBM; mm_reset + mm_post_recvs
++ mm_push_msgs + mm_match_batch are all inside the timed region).
+
+Headline `value`: the MPI-compliant level on configs[1] (4096 endpoints x
+1024-deep receive/message queues, proxy-app src/tag mix, 5% ANY_SOURCE).
+`levels` adds the relaxed levels on their own workloads (configs[2]: 16M
+pairs sort+rank; configs[3]: 32M pairs per GPU hash table, 256M at 8 GPUs).
+Multi-GPU (torchrun): MPI endpoints are split over ranks (weak scaling, no
+collective); the no-wildcard levels shard the tuple key space with
+mm_route + NCCL all-to-all (paper_conf_ipps_klenkfed17_b200/parallel.py).
+
+Rank 0 prints ONE JSON line.  The oracle (oracle/) is only used for the
+cpu_baseline leg and for --impl reference.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "matches/sec per semantics level (device-timed) at 1/2/4/8 B200; HBM GB/s"
+WORKLOADS = {
+    "mpi": "configs[1]: MPI-compliant with wildcards, 4096 endpoints x 1024-deep recv/msg queues, "
+           "proxy-app-shaped src/tag mix (10-30 peers, 1..4096 tags), 5% ANY_SOURCE",
+    "ordered": "configs[2]: no wildcards, per-(src,tag) ordering kept: 16M recv/msg pairs via sort+rank pairing",
+    "unordered": "configs[3]: no wildcards, no ordering: 32M pairs per GPU (256M at 8 GPUs) via hash-table matching",
+}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def load_traffic(kernel):
+    """dram bytes per launch of `kernel` from the committed ncu capture summary."""
+    p = os.path.join(ROOT, "profiles", "kernel_traffic.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        d = json.load(f)
+    v = d.get(kernel)
+    return v.get("dram_bytes_per_launch") if isinstance(v, dict) else None
+
+
+class Clocks:
+    """Samples nvidia-smi clocks / throttle reasons while a region runs."""
+
+    def __init__(self, index=0):
+        self.index = index
+        self.proc = None
+        self.path = os.path.join("/tmp", "mm_clocks_%d_%d.csv" % (os.getpid(), index))
+
+    def start(self):
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + q,
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.f.close()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx.append(float(parts[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        os.unlink(self.path)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm), "window": "warmup+timed steps of every level"}
+
+
+# ----------------------------------------------------------------- workloads
+def mpi_workload(rank):
+    import synth
+    return synth.proxy_endpoints(seed=1 + 1000 * rank)
+
+
+def ordered_workload(rank, world):
+    import synth
+    n = (1 << 24) // world  # configs[2]: 16M pairs in total
+    return synth.nowild_pairs(seed=2 + 1000 * rank, n=n, n_src=1 << 16, n_tag=64)
+
+
+def unordered_workload(rank):
+    import synth
+    return synth.nowild_pairs(seed=3 + 1000 * rank, n=1 << 25, n_src=1 << 20, n_tag=1 << 12)
+
+
+def to_dev(a):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(a).view(np.int64).copy()).cuda()
+
+
+# --------------------------------------------------------------- our levels
+def bench_mpi(args, world, rank, peak):
+    import torch
+
+    import paper_conf_ipps_klenkfed17_b200 as mm
+    q = mpi_workload(rank)
+    n_ep, depth = q.n_endpoints, 1024
+    n_r, n_m = len(q.recv_hdr), len(q.msg_hdr)
+    # 4 rotating copies of the inputs (4 x 64 MB of headers > 126 MB L2)
+    ncopy = 4
+    rh = [to_dev(q.recv_hdr) for _ in range(ncopy)]
+    mh = [to_dev(q.msg_hdr) for _ in range(ncopy)]
+    ro, mo = to_dev(q.recv_off), to_dev(q.msg_off)
+    orc = [torch.empty(n_r, dtype=torch.int64, device="cuda") for _ in range(ncopy)]
+    omc = [torch.empty(n_r, dtype=torch.int64, device="cuda") for _ in range(ncopy)]
+    cnt = [torch.zeros(2, dtype=torch.int64, device="cuda") for _ in range(ncopy)]
+    eng = mm.Engine(mm.MM_SEM_MPI, n_ep, depth, depth)
+
+    def step(i):
+        s = i % ncopy
+        eng.reset()
+        eng.post_recvs(rh[s], None, ro)
+        eng.push_msgs(mh[s], None, mo)
+        eng.match_batch(orc[s], omc[s], cnt[s])
+
+    res = timed(args, step, eng, world)
+    matches = int(cnt[0][1].item())
+    assert all(int(c[1].item()) == matches for c in cnt)
+    q1 = eng.query()
+    resid = q1["resid_recv"] + q1["resid_msg"]
+    # algorithmic bytes of the matcher kernel per launch: every header read
+    # once, (recv cookie, msg cookie) written per receive, survivors compacted
+    algo = 8 * (n_r + n_m) + 16 * n_r + 16 * resid
+    res.update(matches_per_step=matches, algo_bytes=algo, kernel="k_mpi_matrix", n_recv=n_r, n_msg=n_m)
+    res["e2e"] = bench_mpi_e2e(args, q, eng, world)
+    eng.close()
+    return finish_level(res, world, peak, "mpi")
+
+
+def bench_mpi_e2e(args, q, eng, world):
+    """Same metric through the public API with pinned HOST buffers: H2D of the
+    step's inputs and D2H of its result are inside the timed region."""
+    import torch
+    n_r = len(q.recv_hdr)
+    pin = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.int64).copy()).pin_memory()
+    rh, mh = pin(q.recv_hdr), pin(q.msg_hdr)
+    ro, mo = pin(q.recv_off), pin(q.msg_off)
+    orc = torch.empty(n_r, dtype=torch.int64).pin_memory()
+    omc = torch.empty(n_r, dtype=torch.int64).pin_memory()
+    cnt = torch.zeros(2, dtype=torch.int64).pin_memory()
+
+    def step(i):
+        eng.reset()
+        eng.post_recvs(rh, None, ro)
+        eng.push_msgs(mh, None, mo)
+        eng.match_batch(orc, omc, cnt)
+
+    r = timed(args, step, eng, world, query=False)
+    matches = int(cnt[1])
+    h2d = 8 * (len(q.recv_hdr) + len(q.msg_hdr)) + 8 * (len(q.recv_off) + len(q.msg_off))
+    d2h = 16 * n_r + 16
+    tot = matches * world
+    return {"value": tot * args.steps / (r["t_ms"] / 1e3), "unit": "matches/s", "h2d_bytes_per_step": h2d,
+            "d2h_bytes_per_step": d2h, "ms_per_step": r["t_ms"] / args.steps}
+
+
+def bench_flat(args, world, rank, peak, level):
+    import torch
+
+    import paper_conf_ipps_klenkfed17_b200 as mm
+    q = ordered_workload(rank, world) if level == "ordered" else unordered_workload(rank)
+    n = len(q.recv_hdr)
+    sem = mm.MM_SEM_NOWILD_ORDERED if level == "ordered" else mm.MM_SEM_NOWILD_UNORDERED
+    rh, mh = to_dev(q.recv_hdr), to_dev(q.msg_hdr)
+    if world == 1:
+        eng = mm.Engine(sem, 1, n, n)
+        orc = torch.empty(n, dtype=torch.int64, device="cuda")
+        omc = torch.empty(n, dtype=torch.int64, device="cuda")
+        cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+
+        def step(i):
+            eng.reset()
+            eng.post_recvs(rh)
+            eng.push_msgs(mh)
+            eng.match_batch(orc, omc, cnt)
+
+        res = timed(args, step, eng, world)
+        matches = int(cnt[1].item())
+    else:
+        from paper_conf_ipps_klenkfed17_b200 import parallel
+        eng = parallel.ShardedMatcher(sem, capacity=2 * n)
+
+        def step(i):
+            eng.match(rh, mh)
+
+        res = timed(args, step, eng.engine, world)
+        matches = eng.last_local_matches()
+    algo = 8 * 2 * n + 16 * n
+    res.update(matches_per_step=matches, algo_bytes=algo, n_recv=n, n_msg=n,
+               kernel="sort-and-rank kernels" if level == "ordered" else "hash insert+probe kernels")
+    eng.close()
+    return finish_level(res, world, peak, level)
+
+
+def timed(args, step, eng, world, query=True):
+    import torch
+    import torch.distributed as dist
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+    q0 = eng.query() if query else None
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for i in range(args.steps):
+        step(args.warmup + i)
+    e1.record()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    t = e0.elapsed_time(e1)
+    if world > 1:
+        tt = torch.tensor([t], dtype=torch.float64, device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t = float(tt.item())
+    out = {"t_ms": t}
+    if query:
+        q1 = eng.query()
+        runs = max(1, q1["kernel_runs"] - q0["kernel_runs"])
+        out["kernel_ms"] = (q1["kernel_ns"] - q0["kernel_ns"]) / runs / 1e6
+        out["launches"] = q1["launches"] - q0["launches"]
+    return out
+
+
+def finish_level(res, world, peak, level):
+    import torch
+    import torch.distributed as dist
+    matches = res["matches_per_step"]
+    total = matches
+    if world > 1:
+        t = torch.tensor([matches], dtype=torch.int64, device="cuda")
+        dist.all_reduce(t)
+        total = int(t.item())
+    steps = res["steps"] if "steps" in res else None
+    del steps
+    kernel_ms = res.get("kernel_ms")
+    achieved = res["algo_bytes"] / (kernel_ms / 1e3) / 1e9 if kernel_ms else None
+    out = {
+        "value": None, "unit": "matches/s", "workload": WORKLOADS[level],
+        "matches_per_step": total, "ms_per_step": None,
+        "roofline": {"bound": "hbm", "kernel": res["kernel"], "achieved": achieved, "peak": peak[0],
+                     "peak_source": peak[1], "unit": "GB/s",
+                     "frac": (achieved / peak[0]) if achieved else None,
+                     "traffic": load_traffic(res["kernel"]),
+                     "kernel_ms": kernel_ms, "algo_bytes_per_launch": res["algo_bytes"]},
+        "_t_ms": res["t_ms"], "_launches": res.get("launches"),
+    }
+    if "e2e" in res:
+        out["e2e"] = res["e2e"]
+    return out
+
+
+def finalize_values(levels, steps):
+    for lv in levels.values():
+        lv["ms_per_step"] = lv["_t_ms"] / steps
+        lv["value"] = lv["matches_per_step"] * steps / (lv["_t_ms"] / 1e3)
+
+
+# ------------------------------------------------------------ CPU baseline
+def cpu_baseline(target_s=10.0):
+    """The oracle as it stands (single-threaded C, gcc -O2) on a bounded sample
+    of the configs[1] workload (whole endpoints)."""
+    import oracle
+    q = mpi_workload(0)
+    oracle.lib()
+    n_ep = 32
+    while True:
+        sub = q.subset(range(n_ep))
+        t0 = time.perf_counter()
+        mr, _ = oracle.mpi_endpoints(sub)
+        dt = time.perf_counter() - t0
+        if dt * 2 >= target_s or n_ep >= q.n_endpoints:
+            break
+        n_ep = min(q.n_endpoints, int(n_ep * max(2.0, target_s / max(dt, 1e-3) * 0.6)))
+    matches = int((mr >= 0).sum())
+    return {"value": matches / dt, "unit": "matches/s", "cores": 1, "kind": "oracle",
+            "sample": "%d of 4096 configs[1] endpoints (%d matches) in %.2f s, oracle_mpi_endpoints "
+                      "(classic PRQ/UMQ list traversal, 1 thread)" % (n_ep, matches, dt)}
+
+
+def run_reference(args, world, rank):
+    """--impl reference: the CPU oracle, as it stands, on a bounded sample of
+    the headline workload per step (rank 0 only)."""
+    if rank != 0:
+        return
+    import oracle
+    q = mpi_workload(0)
+    oracle.lib()
+    sub = q.subset(range(64))
+    times, matches = [], 0
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        mr, _ = oracle.mpi_endpoints(sub)
+        dt = time.perf_counter() - t0
+        if i >= args.warmup:
+            times.append(dt)
+            matches = int((mr >= 0).sum())
+    t = sum(times)
+    v = matches * args.steps / t
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "matches/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "config": {"workload": WORKLOADS["mpi"], "sample": "64 of 4096 endpoints per step"},
+        "cpu_baseline": {"value": v, "unit": "matches/s", "cores": 1, "kind": "oracle",
+                         "sample": "64 configs[1] endpoints per step, oracle_mpi_endpoints, 1 thread"},
+        "e2e": {"value": v, "unit": "matches/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--levels", default="mpi,ordered,unordered")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(3, args.warmup)
+    world, rank, local = dist_env()
+    if args.impl == "reference":
+        run_reference(args, world, rank)
+        return
+    import torch
+    torch.cuda.set_device(local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    peak = load_peaks()
+    clocks = Clocks(local)
+    clocks.start()
+    levels = {}
+    wanted = args.levels.split(",")
+    if "mpi" in wanted:
+        levels["mpi"] = bench_mpi(args, world, rank, peak)
+    for lv in ("ordered", "unordered"):
+        if lv in wanted:
+            levels[lv] = bench_flat(args, world, rank, peak, lv)
+    ck = clocks.stop()
+    finalize_values(levels, args.steps)
+    head = levels.get("mpi") or next(iter(levels.values()))
+    line = {
+        "metric": METRIC, "value": head["value"], "unit": "matches/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": head["ms_per_step"], "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "config": {"workload": head["workload"], "level": "mpi" if "mpi" in levels else wanted[0],
+                   "l2": "inputs > L2: 4 rotating copies of the configs[1] headers (256 MB); relaxed levels "
+                         "use 256-512 MB inputs", "parallelism": "endpoints split over %d GPU(s)" % world},
+        "roofline": {k: v for k, v in head["roofline"].items()},
+        "e2e": head.get("e2e"),
+        "gpu_launches": head["_launches"],
+        "clocks": ck,
+        "levels": {k: {kk: vv for kk, vv in v.items() if not kk.startswith("_")} for k, v in levels.items()},
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,590 @@
+// mm_engine.cu -- the C-ABI of include/mm.h (host side).
+//
+// Owns the per-endpoint queues in HBM, stages host buffers, and sequences the
+// kernels of k_mpi.cu / k_flat.cu on the engine's stream.  No matching
+// arithmetic happens on the host.
+#include <stdlib.h>
+#include <string.h>
+
+#include <new>
+
+#include "mm_kernels.h"
+
+using namespace mm;
+
+namespace mm {
+long long& launch_count() {
+  static long long n = 0;
+  return n;
+}
+}  // namespace mm
+
+namespace {
+
+// Ring of CUDA event pairs bracketing the dominant kernel region of each
+// mm_match_batch; resolved lazily so timing never blocks the launch stream.
+struct Timer {
+  static constexpr int kRing = 64;
+  cudaEvent_t a[kRing] = {}, b[kRing] = {};
+  int head = 0, count = 0;  // pending pairs: [head - count, head)
+  bool ok = false;
+  long long ns = 0, runs = 0;
+  void init() {
+    ok = true;
+    for (int i = 0; i < kRing; i++)
+      if (cudaEventCreate(&a[i]) != cudaSuccess || cudaEventCreate(&b[i]) != cudaSuccess) ok = false;
+    if (!ok) cudaGetLastError();
+  }
+  void destroy() {
+    for (int i = 0; i < kRing; i++) {
+      if (a[i]) cudaEventDestroy(a[i]);
+      if (b[i]) cudaEventDestroy(b[i]);
+      a[i] = b[i] = nullptr;
+    }
+  }
+  void resolve_one() {
+    int i = (head - count + kRing) % kRing;
+    float ms = 0.f;
+    if (cudaEventSynchronize(b[i]) == cudaSuccess && cudaEventElapsedTime(&ms, a[i], b[i]) == cudaSuccess) {
+      ns += (long long)(ms * 1e6);
+      runs++;
+    } else {
+      cudaGetLastError();
+    }
+    count--;
+  }
+  void resolve_all() {
+    while (count > 0) resolve_one();
+  }
+  void begin(cudaStream_t st) {
+    if (!ok) return;
+    if (count == kRing) resolve_one();
+    cudaEventRecord(a[head], st);
+  }
+  void end(cudaStream_t st) {
+    if (!ok) return;
+    cudaEventRecord(b[head], st);
+    head = (head + 1) % kRing;
+    count++;
+  }
+};
+
+struct DBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+};
+
+cudaError_t ensure(DBuf& b, size_t bytes) {
+  if (bytes == 0) bytes = 16;
+  if (b.bytes >= bytes) return cudaSuccess;
+  if (b.p) cudaFree(b.p);
+  b.p = nullptr;
+  b.bytes = 0;
+  cudaError_t err = cudaMalloc(&b.p, bytes);
+  if (err == cudaSuccess) b.bytes = bytes;
+  return err;
+}
+
+void release(DBuf& b) {
+  if (b.p) cudaFree(b.p);
+  b.p = nullptr;
+  b.bytes = 0;
+}
+
+bool is_device_ptr(const void* p) {
+  if (!p) return false;
+  cudaPointerAttributes at;
+  cudaError_t err = cudaPointerGetAttributes(&at, p);
+  if (err != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+int64_t next_pow2(int64_t x) {
+  int64_t p = 1;
+  while (p < x) p <<= 1;
+  return p;
+}
+
+struct Pending {
+  const uint64_t* hdr = nullptr;
+  const int64_t* cookie = nullptr;
+  const int64_t* off = nullptr;
+  int64_t n = 0;
+  int64_t seq0 = 0;
+  bool active = false;
+};
+
+struct Queue {
+  DBuf hdr[2], cookie[2], len[2];  // ping-pong (the MPI level compacts in place and uses [0] only)
+  DBuf st_hdr, st_cookie, st_off;   // staging for host inputs
+  Pending pend;
+  int64_t seq = 0;
+  int cur = 0;
+  int64_t resid_host = 0;  // exact residual count (single-endpoint levels)
+};
+
+}  // namespace
+
+struct mm_engine {
+  int sem = 0;
+  int n_ep = 1;
+  int64_t rcap = 0, mcap = 0;
+  cudaStream_t st = nullptr;
+  int dev = 0;
+  Queue rq, mq;
+  DBuf out_off, counts_dev, nmatched, err, info;
+  DBuf out_rc_stage, out_mc_stage;
+  // MPI
+  int64_t msg_slots = 0, warp_words = 0;
+  // single-endpoint levels
+  DBuf rflag, mflag, scan;
+  DBuf skey[2], sval[2], rid, run_start, run_rc, part;
+  DBuf owner, rcnt, mcnt, tkey, tval;
+  int64_t T = 0;
+  Timer timer;
+  long long launches = 0;
+};
+
+// Attributes the library's kernel launches during one API call to an engine.
+struct LaunchScope {
+  mm_engine* e;
+  long long start;
+  explicit LaunchScope(mm_engine* en) : e(en), start(mm::launch_count()) {}
+  ~LaunchScope() {
+    if (e) e->launches += mm::launch_count() - start;
+  }
+};
+
+#define CK(x)                                   \
+  do {                                          \
+    cudaError_t _e = (x);                       \
+    if (_e != cudaSuccess) return MM_ERR_CUDA;  \
+  } while (0)
+
+static Side make_side(mm_engine* e, Queue& q, int64_t cap) {
+  Side s;
+  s.q_hdr = (const uint64_t*)q.hdr[q.cur].p;
+  s.q_cookie = (const int64_t*)q.cookie[q.cur].p;
+  s.q_len = (const int32_t*)q.len[q.cur].p;
+  s.p_hdr = q.pend.active ? q.pend.hdr : nullptr;
+  s.p_cookie = q.pend.active ? q.pend.cookie : nullptr;
+  s.p_off = q.pend.active ? q.pend.off : nullptr;
+  s.p_n = q.pend.active ? q.pend.n : 0;
+  s.p_seq0 = q.pend.seq0;
+  s.cap = cap;
+  (void)e;
+  return s;
+}
+
+static int alloc_queue(mm_engine* e, Queue& q, int64_t cap, bool pingpong) {
+  const int64_t slots = (int64_t)e->n_ep * cap;
+  for (int b = 0; b < (pingpong ? 2 : 1); b++) {
+    CK(ensure(q.hdr[b], slots * 8));
+    CK(ensure(q.cookie[b], slots * 8));
+    CK(ensure(q.len[b], (size_t)e->n_ep * 4));
+    CK(cudaMemsetAsync(q.len[b].p, 0, (size_t)e->n_ep * 4, e->st));
+  }
+  return MM_OK;
+}
+
+extern "C" {
+
+const char* mm_strerror(int code) {
+  switch (code) {
+    case MM_OK: return "ok";
+    case MM_ERR_ARG: return "invalid argument";
+    case MM_ERR_CUDA: return "CUDA runtime error";
+    case MM_ERR_CAPACITY: return "queue or output capacity exceeded";
+    case MM_ERR_NOMEM: return "out of memory";
+    case MM_ERR_STATE: return "invalid state";
+    default: return "unknown error";
+  }
+}
+
+const char* mm_version(void) { return "mm 0.1.0 sm_100a"; }
+
+int mm_destroy(mm_engine* e) {
+  if (!e) return MM_OK;
+  cudaStreamSynchronize(e->st);
+  e->timer.destroy();
+  Queue* qs[2] = {&e->rq, &e->mq};
+  for (Queue* q : qs) {
+    for (int b = 0; b < 2; b++) {
+      release(q->hdr[b]);
+      release(q->cookie[b]);
+      release(q->len[b]);
+    }
+    release(q->st_hdr);
+    release(q->st_cookie);
+    release(q->st_off);
+  }
+  DBuf* bufs[] = {&e->out_off, &e->counts_dev, &e->nmatched, &e->err, &e->info, &e->out_rc_stage,
+                  &e->out_mc_stage, &e->rflag, &e->mflag, &e->scan, &e->skey[0], &e->skey[1],
+                  &e->sval[0], &e->sval[1], &e->rid, &e->run_start, &e->run_rc, &e->part,
+                  &e->owner, &e->rcnt, &e->mcnt, &e->tkey, &e->tval};
+  for (DBuf* b : bufs) release(*b);
+  delete e;
+  return MM_OK;
+}
+
+int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t recv_capacity, int64_t msg_capacity,
+              void* stream) {
+  if (!out) return MM_ERR_ARG;
+  *out = nullptr;
+  if (semantics < MM_SEM_MPI || semantics > MM_SEM_NOWILD_UNORDERED) return MM_ERR_ARG;
+  if (n_endpoints < 1 || recv_capacity < 1 || msg_capacity < 1) return MM_ERR_ARG;
+  if (semantics != MM_SEM_MPI && n_endpoints != 1) return MM_ERR_ARG;
+  if (semantics == MM_SEM_MPI && msg_capacity > MM_MPI_MAX_MSGS) return MM_ERR_ARG;
+  if (semantics != MM_SEM_MPI && recv_capacity + msg_capacity >= (int64_t)1 << 31) return MM_ERR_ARG;
+  mm_engine* e = new (std::nothrow) mm_engine();
+  if (!e) return MM_ERR_NOMEM;
+  e->sem = semantics;
+  e->n_ep = n_endpoints;
+  e->rcap = recv_capacity + (recv_capacity & 1);  // even stride keeps 16-byte alignment
+  e->mcap = msg_capacity + (msg_capacity & 1);
+  e->st = (cudaStream_t)stream;
+  if (cudaGetDevice(&e->dev) != cudaSuccess) {
+    cudaGetLastError();
+    delete e;
+    return MM_ERR_CUDA;
+  }
+  int rc = MM_OK;
+  const bool pp = semantics != MM_SEM_MPI;
+  if ((rc = alloc_queue(e, e->rq, e->rcap, pp)) != MM_OK || (rc = alloc_queue(e, e->mq, e->mcap, pp)) != MM_OK) {
+    mm_destroy(e);
+    return rc == MM_ERR_CUDA ? MM_ERR_NOMEM : rc;
+  }
+  bool ok = ensure(e->out_off, (size_t)(n_endpoints + 1) * 8) == cudaSuccess &&
+            ensure(e->counts_dev, 16) == cudaSuccess && ensure(e->nmatched, 8) == cudaSuccess &&
+            ensure(e->err, 4) == cudaSuccess && ensure(e->info, sizeof(SnapInfo)) == cudaSuccess;
+  if (ok && semantics == MM_SEM_MPI) {
+    e->msg_slots = (e->mcap + 63) / 64 * 64;
+    e->warp_words = (e->msg_slots + e->msg_slots / 64 + 3) / 4 * 4;  // headers + availability bits, 32 B aligned
+  }
+  if (ok && semantics != MM_SEM_MPI) {
+    const int64_t n = e->rcap + e->mcap;
+    ok = ensure(e->rflag, e->rcap) == cudaSuccess && ensure(e->mflag, e->mcap) == cudaSuccess &&
+         ensure(e->scan, (size_t)scan_scratch_elems(n) * 8) == cudaSuccess;
+    if (ok && semantics == MM_SEM_NOWILD_ORDERED) {
+      ok = ensure(e->skey[0], n * 8) == cudaSuccess && ensure(e->skey[1], n * 8) == cudaSuccess &&
+           ensure(e->sval[0], n * 4) == cudaSuccess && ensure(e->sval[1], n * 4) == cudaSuccess &&
+           ensure(e->rid, n * 4) == cudaSuccess && ensure(e->run_start, (n + 2) * 4) == cudaSuccess &&
+           ensure(e->run_rc, (n + 2) * 4) == cudaSuccess &&
+           ensure(e->part, (size_t)partition_scratch_elems(n) * 4) == cudaSuccess;
+    }
+    if (ok && semantics == MM_SEM_NOWILD_UNORDERED) {
+      e->T = next_pow2(2 * e->rcap < 1024 ? 1024 : 2 * e->rcap);
+      ok = ensure(e->owner, e->T * 4) == cudaSuccess && ensure(e->rcnt, e->T * 4) == cudaSuccess &&
+           ensure(e->mcnt, e->T * 4) == cudaSuccess && ensure(e->tkey, e->T * 8) == cudaSuccess &&
+           ensure(e->tval, e->T * 4) == cudaSuccess;
+    }
+  }
+  if (!ok) {
+    cudaGetLastError();
+    mm_destroy(e);
+    return MM_ERR_NOMEM;
+  }
+  if (cudaMemsetAsync(e->err.p, 0, 4, e->st) != cudaSuccess) {
+    mm_destroy(e);
+    return MM_ERR_CUDA;
+  }
+  e->timer.init();
+  *out = e;
+  return MM_OK;
+}
+
+static int materialize(mm_engine* e, Queue& q, int64_t cap) {
+  if (!q.pend.active) return MM_OK;
+  Side s = make_side(e, q, cap);
+  CK(launch_materialize(s, e->n_ep, (uint64_t*)q.hdr[q.cur].p, (int64_t*)q.cookie[q.cur].p, (int32_t*)q.len[q.cur].p,
+                        (uint32_t*)e->err.p, e->st));
+  q.resid_host += q.pend.n;
+  if (q.resid_host > cap) q.resid_host = cap;
+  q.pend = Pending();
+  return MM_OK;
+}
+
+static int post(mm_engine* e, Queue& q, int64_t cap, const uint64_t* hdr, const int64_t* cookie,
+                const int64_t* off, int64_t n) {
+  if (!e || n < 0 || (n > 0 && !hdr)) return MM_ERR_ARG;
+  if (e->n_ep > 1 && !off) return MM_ERR_ARG;
+  const bool off_dev = is_device_ptr(off);
+  if (off && !off_dev) {  // host offsets can be validated here
+    if (off[0] != 0 || off[e->n_ep] != n) return MM_ERR_ARG;
+    for (int i = 0; i < e->n_ep; i++)
+      if (off[i + 1] < off[i]) return MM_ERR_ARG;
+  }
+  int rc = materialize(e, q, cap);
+  if (rc != MM_OK) return rc;
+  Pending p;
+  p.n = n;
+  p.seq0 = q.seq;
+  p.active = n > 0;
+  if (n > 0) {
+    if (is_device_ptr(hdr)) {
+      p.hdr = hdr;
+    } else {
+      CK(ensure(q.st_hdr, (size_t)n * 8));
+      CK(cudaMemcpyAsync(q.st_hdr.p, hdr, (size_t)n * 8, cudaMemcpyHostToDevice, e->st));
+      p.hdr = (const uint64_t*)q.st_hdr.p;
+    }
+    if (cookie) {
+      if (is_device_ptr(cookie)) {
+        p.cookie = cookie;
+      } else {
+        CK(ensure(q.st_cookie, (size_t)n * 8));
+        CK(cudaMemcpyAsync(q.st_cookie.p, cookie, (size_t)n * 8, cudaMemcpyHostToDevice, e->st));
+        p.cookie = (const int64_t*)q.st_cookie.p;
+      }
+    }
+    if (off) {
+      if (off_dev) {
+        p.off = off;
+      } else {
+        CK(ensure(q.st_off, (size_t)(e->n_ep + 1) * 8));
+        CK(cudaMemcpyAsync(q.st_off.p, off, (size_t)(e->n_ep + 1) * 8, cudaMemcpyHostToDevice, e->st));
+        p.off = (const int64_t*)q.st_off.p;
+      }
+    }
+  }
+  q.seq += n;
+  q.pend = p;
+  return MM_OK;
+}
+
+int mm_post_recvs(mm_engine* e, const uint64_t* hdr, const int64_t* cookie, const int64_t* ep_offsets, int64_t n) {
+  if (!e) return MM_ERR_ARG;
+  LaunchScope ls(e);
+  return post(e, e->rq, e->rcap, hdr, cookie, ep_offsets, n);
+}
+
+int mm_push_msgs(mm_engine* e, const uint64_t* hdr, const int64_t* cookie, const int64_t* ep_offsets, int64_t n) {
+  if (!e) return MM_ERR_ARG;
+  LaunchScope ls(e);
+  return post(e, e->mq, e->mcap, hdr, cookie, ep_offsets, n);
+}
+
+int mm_reset(mm_engine* e) {
+  if (!e) return MM_ERR_ARG;
+  Queue* qs[2] = {&e->rq, &e->mq};
+  for (Queue* q : qs) {
+    for (int b = 0; b < 2; b++)
+      if (q->len[b].p) CK(cudaMemsetAsync(q->len[b].p, 0, (size_t)e->n_ep * 4, e->st));
+    q->pend = Pending();
+    q->seq = 0;
+    q->cur = 0;
+    q->resid_host = 0;
+  }
+  CK(cudaMemsetAsync(e->err.p, 0, 4, e->st));
+  return MM_OK;
+}
+
+// Copy device outputs to host outputs / counts when the caller passed host memory.
+static int deliver(mm_engine* e, int64_t* out_rc, int64_t* out_mc, bool host_out, int64_t n_copy, int64_t* counts,
+                   bool counts_host) {
+  if (host_out && n_copy > 0) {
+    CK(cudaMemcpyAsync(out_rc, e->out_rc_stage.p, (size_t)n_copy * 8, cudaMemcpyDeviceToHost, e->st));
+    CK(cudaMemcpyAsync(out_mc, e->out_mc_stage.p, (size_t)n_copy * 8, cudaMemcpyDeviceToHost, e->st));
+  }
+  if (counts && counts_host) CK(cudaMemcpyAsync(counts, e->counts_dev.p, 16, cudaMemcpyDeviceToHost, e->st));
+  if (host_out || (counts && counts_host)) CK(cudaStreamSynchronize(e->st));
+  return MM_OK;
+}
+
+static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out_cap, int64_t* counts) {
+  const bool host_out = !is_device_ptr(out_rc) || !is_device_ptr(out_mc);
+  const bool counts_host = counts && !is_device_ptr(counts);
+  int64_t* drc = out_rc;
+  int64_t* dmc = out_mc;
+  if (host_out) {
+    CK(ensure(e->out_rc_stage, (size_t)out_cap * 8));
+    CK(ensure(e->out_mc_stage, (size_t)out_cap * 8));
+    drc = (int64_t*)e->out_rc_stage.p;
+    dmc = (int64_t*)e->out_mc_stage.p;
+  }
+  Side R = make_side(e, e->rq, e->rcap), M = make_side(e, e->mq, e->mcap);
+  CK(cudaMemsetAsync(e->nmatched.p, 0, 8, e->st));
+  CK(launch_out_offsets(R, e->n_ep, (int64_t*)e->out_off.p, out_cap, (uint32_t*)e->err.p, e->st));
+  MpiArgs a;
+  a.R = R;
+  a.M = M;
+  a.n_ep = e->n_ep;
+  a.msg_slots = e->msg_slots;
+  a.warp_smem_words = e->warp_words;
+  a.out_rc = drc;
+  a.out_mc = dmc;
+  a.out_cap = out_cap;
+  a.out_off = (const int64_t*)e->out_off.p;
+  a.q_rh_w = (uint64_t*)e->rq.hdr[0].p;
+  a.q_rc_w = (int64_t*)e->rq.cookie[0].p;
+  a.rres_w = (int32_t*)e->rq.len[0].p;
+  a.q_mh_w = (uint64_t*)e->mq.hdr[0].p;
+  a.q_mc_w = (int64_t*)e->mq.cookie[0].p;
+  a.mres_w = (int32_t*)e->mq.len[0].p;
+  a.n_matched = (unsigned long long*)e->nmatched.p;
+  a.err = (uint32_t*)e->err.p;
+  e->timer.begin(e->st);
+  CK(launch_mpi_matrix(a, e->st));
+  e->timer.end(e->st);
+  CK(launch_finalize((const int64_t*)e->out_off.p + e->n_ep, 0, (const unsigned long long*)e->nmatched.p,
+                     (int64_t*)e->counts_dev.p, e->st));
+  e->rq.pend = Pending();
+  e->mq.pend = Pending();
+  if (counts && !counts_host) CK(cudaMemcpyAsync(counts, e->counts_dev.p, 16, cudaMemcpyDeviceToDevice, e->st));
+  int64_t n_copy = 0;
+  if (host_out) {
+    // the snapshot size is only known on the device: fetch it first
+    int64_t tot = 0;
+    CK(cudaMemcpyAsync(&tot, (const int64_t*)e->out_off.p + e->n_ep, 8, cudaMemcpyDeviceToHost, e->st));
+    CK(cudaStreamSynchronize(e->st));
+    n_copy = tot < out_cap ? tot : out_cap;
+  }
+  return deliver(e, out_rc, out_mc, host_out, n_copy, counts, counts_host);
+}
+
+static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out_cap, int64_t* counts) {
+  const bool host_out = !is_device_ptr(out_rc) || !is_device_ptr(out_mc);
+  const bool counts_host = counts && !is_device_ptr(counts);
+  const bool ordered = e->sem == MM_SEM_NOWILD_ORDERED;
+  Side R = make_side(e, e->rq, e->rcap), M = make_side(e, e->mq, e->mcap);
+  // exact residual sizes (and, for the sort, the varying header bits)
+  const int64_t bound = e->rq.resid_host + R.p_n + e->mq.resid_host + M.p_n;
+  CK(launch_snapshot_info(R, M, bound, (SnapInfo*)e->info.p, ordered, e->st));
+  SnapInfo info;
+  CK(cudaMemcpyAsync(&info, e->info.p, sizeof(SnapInfo), cudaMemcpyDeviceToHost, e->st));
+  CK(cudaStreamSynchronize(e->st));
+  const int64_t nr = info.rres + R.p_n, nm = info.mres + M.p_n;
+  if (nr > e->rcap || nm > e->mcap) return MM_ERR_CAPACITY;
+  if (nr > out_cap) return MM_ERR_CAPACITY;
+  int64_t* drc = out_rc;
+  int64_t* dmc = out_mc;
+  if (host_out) {
+    CK(ensure(e->out_rc_stage, (size_t)(nr > 0 ? nr : 1) * 8));
+    CK(ensure(e->out_mc_stage, (size_t)(nr > 0 ? nr : 1) * 8));
+    drc = (int64_t*)e->out_rc_stage.p;
+    dmc = (int64_t*)e->out_mc_stage.p;
+  }
+  CK(cudaMemsetAsync(e->nmatched.p, 0, 8, e->st));
+  FlatArgs a;
+  a.R = R;
+  a.M = M;
+  a.nr = nr;
+  a.nm = nm;
+  a.n_matched = (unsigned long long*)e->nmatched.p;
+  a.out_rc = drc;
+  a.out_mc = dmc;
+  a.rflag = (uint8_t*)e->rflag.p;
+  a.mflag = (uint8_t*)e->mflag.p;
+  if (ordered) {
+    SortScratch s;
+    for (int b = 0; b < 2; b++) {
+      s.key[b] = (uint64_t*)e->skey[b].p;
+      s.val[b] = (uint32_t*)e->sval[b].p;
+    }
+    s.rid = (uint32_t*)e->rid.p;
+    s.run_start = (uint32_t*)e->run_start.p;
+    s.run_rc = (uint32_t*)e->run_rc.p;
+    s.part = (uint32_t*)e->part.p;
+    s.scan = (unsigned long long*)e->scan.p;
+    e->timer.begin(e->st);
+    CK(run_sort_rank(a, info.ref, info.diff, s, e->st));
+    e->timer.end(e->st);
+  } else {
+    HashScratch h;
+    h.owner = (uint32_t*)e->owner.p;
+    h.rcnt = (uint32_t*)e->rcnt.p;
+    h.mcnt = (uint32_t*)e->mcnt.p;
+    h.tkey = (unsigned long long*)e->tkey.p;
+    h.tval = (uint32_t*)e->tval.p;
+    h.T = next_pow2(2 * nr < 1024 ? 1024 : 2 * nr);
+    e->timer.begin(e->st);
+    CK(run_hash(a, h, e->st));
+    e->timer.end(e->st);
+  }
+  // compact both queues into the other ping-pong buffer
+  Queue* qs[2] = {&e->rq, &e->mq};
+  const Side* ss[2] = {&R, &M};
+  const int64_t ns[2] = {nr, nm};
+  const int64_t res[2] = {info.rres, info.mres};
+  const uint8_t* fl[2] = {a.rflag, a.mflag};
+  for (int i = 0; i < 2; i++) {
+    Queue& q = *qs[i];
+    const int nb = q.cur ^ 1;
+    CK(run_compact(*ss[i], res[i], ns[i], fl[i], (uint64_t*)q.hdr[nb].p, (int64_t*)q.cookie[nb].p,
+                   (int32_t*)q.len[nb].p, (uint32_t*)e->scan.p, e->st));
+    q.cur = nb;
+    q.pend = Pending();
+    q.resid_host = ns[i];  // upper bound until the next exact read
+  }
+  CK(launch_finalize(nullptr, nr, (const unsigned long long*)e->nmatched.p, (int64_t*)e->counts_dev.p, e->st));
+  if (counts && !counts_host) CK(cudaMemcpyAsync(counts, e->counts_dev.p, 16, cudaMemcpyDeviceToDevice, e->st));
+  return deliver(e, out_rc, out_mc, host_out, nr < out_cap ? nr : out_cap, counts, counts_host);
+}
+
+int mm_match_batch(mm_engine* e, int64_t* out_recv_cookie, int64_t* out_msg_cookie, int64_t out_capacity,
+                   int64_t* counts) {
+  if (!e || out_capacity < 0 || (out_capacity > 0 && (!out_recv_cookie || !out_msg_cookie))) return MM_ERR_ARG;
+  LaunchScope ls(e);
+  if (e->sem == MM_SEM_MPI) return match_mpi(e, out_recv_cookie, out_msg_cookie, out_capacity, counts);
+  return match_flat(e, out_recv_cookie, out_msg_cookie, out_capacity, counts);
+}
+
+int mm_query(mm_engine* e, int64_t* vals) {
+  if (!e || !vals) return MM_ERR_ARG;
+  CK(cudaStreamSynchronize(e->st));
+  int64_t c[2] = {0, 0};
+  CK(cudaMemcpy(c, e->counts_dev.p, 16, cudaMemcpyDeviceToHost));
+  uint32_t err = 0;
+  CK(cudaMemcpy(&err, e->err.p, 4, cudaMemcpyDeviceToHost));
+  int64_t rsum = 0, msum = 0;
+  int32_t* tmp = (int32_t*)malloc((size_t)e->n_ep * 4);
+  if (!tmp) return MM_ERR_NOMEM;
+  CK(cudaMemcpy(tmp, e->rq.len[e->rq.cur].p, (size_t)e->n_ep * 4, cudaMemcpyDeviceToHost));
+  for (int i = 0; i < e->n_ep; i++) rsum += tmp[i];
+  CK(cudaMemcpy(tmp, e->mq.len[e->mq.cur].p, (size_t)e->n_ep * 4, cudaMemcpyDeviceToHost));
+  for (int i = 0; i < e->n_ep; i++) msum += tmp[i];
+  free(tmp);
+  vals[MM_Q_N_OUT] = c[0];
+  vals[MM_Q_N_MATCHED] = c[1];
+  vals[MM_Q_RESID_RECV] = rsum;
+  vals[MM_Q_RESID_MSG] = msum;
+  vals[MM_Q_ERROR] = err;
+  e->timer.resolve_all();
+  vals[MM_Q_KERNEL_NS] = e->timer.ns;
+  vals[MM_Q_KERNEL_RUNS] = e->timer.runs;
+  vals[MM_Q_LAUNCHES] = e->launches;
+  if (e->sem != MM_SEM_MPI) {
+    e->rq.resid_host = rsum;
+    e->mq.resid_host = msum;
+  }
+  return err ? MM_ERR_CAPACITY : MM_OK;
+}
+
+int mm_route(const uint64_t* a, const int64_t* b, int64_t n, int32_t world, int32_t by, uint64_t* out_a,
+             int64_t* out_b, int64_t* counts, void* stream) {
+  if (n < 0 || world < 1 || world > 256 || (by != 0 && by != 1)) return MM_ERR_ARG;
+  if (n > 0 && (!a || !out_a || !out_b)) return MM_ERR_ARG;
+  if (!counts) return MM_ERR_ARG;
+  if (n >= ((int64_t)1 << 32)) return MM_ERR_ARG;
+  cudaStream_t st = (cudaStream_t)stream;
+  if (n > 0 && (!is_device_ptr(a) || !is_device_ptr(out_a) || !is_device_ptr(out_b) || (b && !is_device_ptr(b))))
+    return MM_ERR_ARG;
+  const bool counts_host = !is_device_ptr(counts);
+  void* part = nullptr;
+  void* dcounts = nullptr;
+  CK(cudaMallocAsync(&part, (size_t)partition_scratch_elems(n > 0 ? n : 1) * 4, st));
+  CK(cudaMallocAsync(&dcounts, (size_t)world * 8, st));
+  cudaError_t err = run_route(a, b, n, world, by, out_a, out_b, (int64_t*)dcounts, (uint32_t*)part, st);
+  if (err == cudaSuccess)
+    err = cudaMemcpyAsync(counts, dcounts, (size_t)world * 8,
+                          counts_host ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice, st);
+  cudaFreeAsync(part, st);
+  cudaFreeAsync(dcounts, st);
+  if (err == cudaSuccess && counts_host) err = cudaStreamSynchronize(st);
+  return err == cudaSuccess ? MM_OK : MM_ERR_CUDA;
+}
+
+}  // extern "C"

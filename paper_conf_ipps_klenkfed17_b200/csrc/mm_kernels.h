@@ -1,0 +1,90 @@
+// mm_kernels.h -- argument blocks and launchers of the matching kernels.
+#pragma once
+
+#include "mm_internal.cuh"
+
+namespace mm {
+
+struct MpiArgs {
+  Side R, M;
+  int n_ep;
+  int64_t msg_slots;        // shared-memory message slots per warp (>= msg cap, multiple of 64)
+  int64_t warp_smem_words;  // 8-byte words of shared memory per warp
+  int64_t* out_rc;
+  int64_t* out_mc;
+  int64_t out_cap;
+  const int64_t* out_off;
+  uint64_t* q_rh_w;
+  int64_t* q_rc_w;
+  int32_t* rres_w;
+  uint64_t* q_mh_w;
+  int64_t* q_mc_w;
+  int32_t* mres_w;
+  unsigned long long* n_matched;
+  uint32_t* err;
+};
+
+cudaError_t launch_out_offsets(const Side& R, int n_ep, int64_t* out_off, int64_t out_cap, uint32_t* err,
+                               cudaStream_t st);
+cudaError_t launch_mpi_matrix(const MpiArgs& a, cudaStream_t st);
+
+// Append the pending elements of every endpoint to its queue (used when a
+// second post/push arrives before a match).
+cudaError_t launch_materialize(const Side& S, int n_ep, uint64_t* q_h, int64_t* q_c, int32_t* q_len, uint32_t* err,
+                               cudaStream_t st);
+
+// ------------------------------------------------- no-wildcard levels (n_ep = 1)
+struct FlatArgs {
+  Side R, M;
+  int64_t nr, nm;  // exact snapshot sizes (host-known)
+  unsigned long long* n_matched;
+  int64_t* out_rc;
+  int64_t* out_mc;
+  uint8_t* rflag;  // 1 = receive matched
+  uint8_t* mflag;  // 1 = message matched
+};
+
+struct SnapInfo {
+  unsigned long long diff;  // OR over all snapshot headers of (hdr ^ ref)
+  unsigned long long ref;
+  int32_t rres, mres;
+};
+cudaError_t launch_snapshot_info(const Side& R, const Side& M, int64_t bound, SnapInfo* info, bool want_diff,
+                                 cudaStream_t st);
+
+// Ordered level: sort-and-rank pairing (row A4).
+struct SortScratch {
+  uint64_t* key[2];
+  uint32_t* val[2];
+  uint32_t* rid;
+  uint32_t* run_start;
+  uint32_t* run_rc;
+  uint32_t* part;  // partition scratch
+  unsigned long long* scan;
+};
+cudaError_t run_sort_rank(const FlatArgs& a, uint64_t ref, uint64_t diff, const SortScratch& s, cudaStream_t st);
+
+// Unordered level: lock-free open-addressing hash table (row A5).
+struct HashScratch {
+  uint32_t* owner;  // [T] receive index owning the slot (EMPTY = 0xFFFFFFFF)
+  uint32_t* rcnt;   // [T] receives with the slot's tuple
+  uint32_t* mcnt;   // [T] messages that probed the slot
+  unsigned long long* tkey;  // [T] ticket table keys (slot << 32 | ticket)
+  uint32_t* tval;            // [T] receive index of a ticket
+  int64_t T;                 // power of two
+};
+cudaError_t run_hash(const FlatArgs& a, const HashScratch& h, cudaStream_t st);
+
+// Compaction of the no-wildcard queues into the other ping-pong buffer.
+cudaError_t run_compact(const Side& S, int64_t resid, int64_t n, const uint8_t* matched, uint64_t* q_h, int64_t* q_c,
+                        int32_t* q_len, uint32_t* scan, cudaStream_t st);
+
+// mm_route
+cudaError_t run_route(const uint64_t* a, const int64_t* b, int64_t n, int world, int by, uint64_t* out_a,
+                      int64_t* out_b, int64_t* counts, uint32_t* part, cudaStream_t st);
+
+// counts[] = {n_out, n_matched} from device state
+cudaError_t launch_finalize(const int64_t* n_out_src, int64_t n_out_host, const unsigned long long* n_matched,
+                            int64_t* counts, cudaStream_t st);
+
+}  // namespace mm

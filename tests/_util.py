@@ -1,0 +1,119 @@
+"""Helpers shared by the parity tests: drive the CUDA path and the oracle on
+the same seeded synth.Queues and compare."""
+from collections import Counter
+
+import numpy as np
+
+import oracle
+
+
+def to_dev(a):
+    import torch
+    if a is None:
+        return None
+    a = np.ascontiguousarray(a)
+    if a.dtype == np.uint64:
+        a = a.view(np.int64)
+    return torch.from_numpy(a.copy()).cuda()
+
+
+def gpu_batches(sem, n_ep, rcap, mcap, batches, host=False, out_cap=None):
+    """batches: list of (recv_hdr, recv_cookie, recv_off, msg_hdr, msg_cookie, msg_off).
+    Returns a list of (out_rc, out_mc) numpy arrays, one per batch."""
+    import torch
+    from paper_conf_ipps_klenkfed17_b200 import Engine
+    eng = Engine(sem, n_ep, rcap, mcap)
+    res = []
+    for (rh, rc, ro, mh, mc, mo) in batches:
+        if host:
+            eng.post_recvs(np.ascontiguousarray(rh, np.uint64), rc, ro)
+            eng.push_msgs(np.ascontiguousarray(mh, np.uint64), mc, mo)
+        else:
+            eng.post_recvs(to_dev(rh), to_dev(rc), to_dev(ro))
+            eng.push_msgs(to_dev(mh), to_dev(mc), to_dev(mo))
+        cap = out_cap if out_cap is not None else n_ep * rcap
+        if host:
+            orc = np.full(cap, -7, np.int64)
+            omc = np.full(cap, -7, np.int64)
+            cnt = np.zeros(2, np.int64)
+            eng.match_batch(orc, omc, cnt)
+            n = int(cnt[0])
+            res.append((orc[:n].copy(), omc[:n].copy(), cnt.copy()))
+        else:
+            orc = torch.full((cap,), -7, dtype=torch.int64, device="cuda")
+            omc = torch.full((cap,), -7, dtype=torch.int64, device="cuda")
+            cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+            eng.match_batch(orc, omc, cnt)
+            torch.cuda.synchronize()
+            c = cnt.cpu().numpy()
+            n = int(c[0])
+            res.append((orc[:n].cpu().numpy(), omc[:n].cpu().numpy(), c))
+    q = eng.query(raise_on_error=False)
+    eng.close()
+    return res, q
+
+
+def oracle_batches(sem, n_ep, batches):
+    eng = oracle.OracleEngine(sem, n_ep)
+    res = []
+    for (rh, rc, ro, mh, mc, mo) in batches:
+        eng.post_recvs(rh, rc, ro)
+        eng.push_msgs(mh, mc, mo)
+        res.append(eng.match_batch())
+    return res, eng
+
+
+def single_batch(q):
+    return [(q.recv_hdr, None, q.recv_off, q.msg_hdr, None, q.msg_off)]
+
+
+def split_batches(q, k, rng):
+    """Split every endpoint's queues into k consecutive pieces at random cuts."""
+    out = []
+    cuts_r = [np.sort(rng.integers(q.recv_off[e], q.recv_off[e + 1] + 1, k - 1)) for e in range(q.n_endpoints)]
+    cuts_m = [np.sort(rng.integers(q.msg_off[e], q.msg_off[e + 1] + 1, k - 1)) for e in range(q.n_endpoints)]
+    for b in range(k):
+        def piece(off, cuts, hdr):
+            hs, cs, o = [], [], [0]
+            for e in range(q.n_endpoints):
+                bounds = [off[e], *cuts[e], off[e + 1]]
+                lo, hi = int(bounds[b]), int(bounds[b + 1])
+                hs.append(hdr[lo:hi]); cs.append(np.arange(lo, hi, dtype=np.int64)); o.append(o[-1] + hi - lo)
+            return np.concatenate(hs).astype(np.uint64), np.concatenate(cs), np.array(o, np.int64)
+        rh, rc, ro = piece(q.recv_off, cuts_r, q.recv_hdr)
+        mh, mc, mo = piece(q.msg_off, cuts_m, q.msg_hdr)
+        out.append((rh, rc, ro, mh, mc, mo))
+    return out
+
+
+def check_unordered(recv_hdr_by_cookie, msg_hdr_by_cookie, out_rc, out_mc, expect_per_key=None):
+    """Validity of an unordered result: matched pairs have equal tuples, each
+    message used at most once, and (if given) per-tuple match counts equal."""
+    m = out_mc >= 0
+    rk = recv_hdr_by_cookie[out_rc[m]]
+    mk = msg_hdr_by_cookie[out_mc[m]]
+    assert np.array_equal(rk, mk), "matched tuples differ"
+    assert len(np.unique(out_mc[m])) == int(m.sum()), "a message matched twice"
+    if expect_per_key is not None:
+        keys, cnt = np.unique(rk, return_counts=True)
+        got = dict(zip(keys.tolist(), cnt.tolist()))
+        assert got == expect_per_key
+
+
+def per_key_min(recv_hdr, msg_hdr):
+    cr = Counter(recv_hdr.tolist())
+    cm = Counter(msg_hdr.tolist())
+    out = {}
+    for k in cr:
+        v = min(cr[k], cm.get(k, 0))
+        if v:
+            out[k] = v
+    return out
+
+
+def per_key_min_np(recv_hdr, msg_hdr):
+    """Vectorised per-key min(#recv, #msg) as (keys, counts) arrays."""
+    ku, cu = np.unique(recv_hdr, return_counts=True)
+    km, cm = np.unique(msg_hdr, return_counts=True)
+    common, ia, ib = np.intersect1d(ku, km, assume_unique=True, return_indices=True)
+    return common, np.minimum(cu[ia], cm[ib])

@@ -1,0 +1,291 @@
+"""Parity of the CUDA path (through the C-ABI) with the CPU oracle.
+
+MPI and NOWILD_ORDERED: bit-exact, element by element (receive cookie and
+matched message cookie for every snapshot receive, per batch).
+NOWILD_UNORDERED: what is unique (reading R6) -- equal tuples per
+pair, every message used once, per-tuple counts equal to the oracle's.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from _util import (check_unordered, gpu_batches, oracle_batches, per_key_min, per_key_min_np, single_batch,
+                   split_batches)
+
+pytestmark = pytest.mark.gpu
+
+MPI, ORD, UNO = oracle.SEM_MPI, oracle.SEM_NOWILD_ORDERED, oracle.SEM_NOWILD_UNORDERED
+
+
+def assert_exact(g, o):
+    assert len(g) == len(o)
+    for b, ((grc, gmc, cnt), (orc, omc)) in enumerate(zip(g, o)):
+        assert len(grc) == len(orc), "batch %d: snapshot sizes differ" % b
+        assert np.array_equal(grc, orc), "batch %d: receive order differs" % b
+        bad = np.nonzero(gmc != omc)[0]
+        assert len(bad) == 0, "batch %d: %d mismatches, first at %s: gpu %s oracle %s" % (
+            b, len(bad), bad[:5], gmc[bad[:5]], omc[bad[:5]])
+        assert int(cnt[1]) == int((omc >= 0).sum())
+
+
+def test_mpi_config0():
+    q = synth.mpi_small(0)
+    g, _ = gpu_batches(MPI, 1, 64, 64, single_batch(q))
+    o, _ = oracle_batches(MPI, 1, single_batch(q))
+    assert_exact(g, o)
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("depth", [1, 31, 33, 200, 1024])
+def test_mpi_ragged_endpoints(seed, depth):
+    q = synth.mpi_endpoints(seed, n_ep=37, depth_r=depth, n_src=5, n_tag=4, p_any_src=0.3, p_any_tag=0.3,
+                            n_comm=2, ragged=True, p_unmatched=0.2)
+    g, qs = gpu_batches(MPI, q.n_endpoints, depth, depth, single_batch(q))
+    o, _ = oracle_batches(MPI, q.n_endpoints, single_batch(q))
+    assert_exact(g, o)
+    assert qs["error"] == 0
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_mpi_multibatch_residuals(seed):
+    rng = np.random.default_rng(seed)
+    q = synth.mpi_endpoints(seed + 10, n_ep=50, depth_r=150, n_src=4, n_tag=3, p_any_src=0.25, p_any_tag=0.25,
+                            ragged=True, p_unmatched=0.3)
+    batches = split_batches(q, 4, rng)
+    g, qs = gpu_batches(MPI, q.n_endpoints, 600, 600, batches)
+    o, oe = oracle_batches(MPI, q.n_endpoints, batches)
+    assert_exact(g, o)
+    rr, rm = oe.residual_depths()
+    assert qs["resid_recv"] == sum(rr) and qs["resid_msg"] == sum(rm)
+
+
+def test_mpi_host_buffers_equal_device():
+    q = synth.mpi_endpoints(5, n_ep=64, depth_r=128, ragged=True, p_unmatched=0.1)
+    gd, _ = gpu_batches(MPI, q.n_endpoints, 128, 128, single_batch(q))
+    gh, _ = gpu_batches(MPI, q.n_endpoints, 128, 128, single_batch(q), host=True)
+    o, _ = oracle_batches(MPI, q.n_endpoints, single_batch(q))
+    assert_exact(gd, o)
+    assert_exact(gh, o)
+
+
+def test_mpi_user_cookies_and_two_posts():
+    """Cookies are carried through; a second post before a match is queued."""
+    q = synth.mpi_endpoints(6, n_ep=8, depth_r=64, p_unmatched=0.1)
+    rng = np.random.default_rng(0)
+    rc = rng.integers(0, 1 << 50, len(q.recv_hdr))
+    mc = rng.integers(0, 1 << 50, len(q.msg_hdr))
+    half_r = q.recv_off // 2
+    # post each endpoint's first half, then the second half, then match once
+    def halves(off, hdr, ck):
+        a_idx = np.concatenate([np.arange(off[e], off[e] + (off[e + 1] - off[e]) // 2) for e in range(8)])
+        b_idx = np.concatenate([np.arange(off[e] + (off[e + 1] - off[e]) // 2, off[e + 1]) for e in range(8)])
+        ao = np.r_[0, np.cumsum([(off[e + 1] - off[e]) // 2 for e in range(8)])]
+        bo = np.r_[0, np.cumsum([(off[e + 1] - off[e]) - (off[e + 1] - off[e]) // 2 for e in range(8)])]
+        return (hdr[a_idx], ck[a_idx], ao), (hdr[b_idx], ck[b_idx], bo)
+    (ra, rb) = halves(q.recv_off, q.recv_hdr, rc)
+    (ma, mb) = halves(q.msg_off, q.msg_hdr, mc)
+    del half_r
+    import torch
+    from _util import to_dev
+    from paper_conf_ipps_klenkfed17_b200 import Engine
+    eng = Engine(MPI, 8, 64, 64)
+    eng.post_recvs(to_dev(ra[0]), to_dev(ra[1]), to_dev(ra[2]))
+    eng.push_msgs(to_dev(ma[0]), to_dev(ma[1]), to_dev(ma[2]))
+    eng.post_recvs(to_dev(rb[0]), to_dev(rb[1]), to_dev(rb[2]))
+    eng.push_msgs(to_dev(mb[0]), to_dev(mb[1]), to_dev(mb[2]))
+    orc = torch.empty(8 * 64, dtype=torch.int64, device="cuda")
+    omc = torch.empty_like(orc)
+    cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+    eng.match_batch(orc, omc, cnt)
+    n = int(cnt[0])
+    oe = oracle.OracleEngine(MPI, 8)
+    oe.post_recvs(*ra)
+    oe.push_msgs(*ma)
+    oe.post_recvs(*rb)
+    oe.push_msgs(*mb)
+    o_rc, o_mc = oe.match_batch()
+    assert np.array_equal(orc[:n].cpu().numpy(), o_rc)
+    assert np.array_equal(omc[:n].cpu().numpy(), o_mc)
+    eng.close()
+
+
+def test_mpi_empty_and_degenerate():
+    # no receives at all, no messages at all, both empty
+    for nr, nm in [(0, 10), (10, 0), (0, 0)]:
+        rh = synth.pack(np.arange(nr) % 3, np.zeros(nr, int))
+        mh = synth.pack(np.arange(nm) % 3, np.zeros(nm, int))
+        b = [(rh, None, np.array([0, nr]), mh, None, np.array([0, nm]))]
+        g, _ = gpu_batches(MPI, 1, 16, 16, b)
+        o, _ = oracle_batches(MPI, 1, b)
+        assert_exact(g, o)
+    # all (ANY, ANY) receives against many senders
+    rh = synth.pack(np.full(100, synth.ANY_SOURCE), np.full(100, synth.ANY_TAG))
+    mh = synth.pack(np.arange(90) % 7, np.arange(90) % 5)
+    b = [(rh, None, np.array([0, 100]), mh, None, np.array([0, 90]))]
+    g, _ = gpu_batches(MPI, 1, 128, 128, b)
+    o, _ = oracle_batches(MPI, 1, b)
+    assert_exact(g, o)
+
+
+def test_mpi_capacity_overflow_is_flagged():
+    q = synth.mpi_endpoints(3, n_ep=4, depth_r=40)
+    g, qs = gpu_batches(MPI, 4, 32, 32, single_batch(q), out_cap=4 * 40)
+    assert qs["error"] != 0 and qs["rc"] == 3
+
+
+def test_mpi_config4_worst_chain():
+    q = synth.worst_chain()
+    g, _ = gpu_batches(MPI, 1, 16384, 16384, single_batch(q))
+    o, _ = oracle_batches(MPI, 1, single_batch(q))
+    assert_exact(g, o)
+
+
+@pytest.mark.slow
+def test_mpi_config1_full():
+    q = synth.proxy_endpoints()
+    g, qs = gpu_batches(MPI, q.n_endpoints, 1024, 1024, single_batch(q))
+    mr, _ = oracle.mpi_endpoints(q)
+    grc, gmc, cnt = g[0]
+    assert np.array_equal(grc, np.arange(len(q.recv_hdr)))
+    assert np.array_equal(gmc, mr), "mismatches: %d" % int((gmc != mr).sum())
+    assert int(cnt[1]) == int((mr >= 0).sum())
+
+
+# ------------------------------------------------------------- relaxations
+
+
+@pytest.mark.parametrize("seed", range(5))
+@pytest.mark.parametrize("n", [1, 100, 4095, 4097, 50000])
+def test_ordered_random(seed, n):
+    q = synth.nowild_pairs(seed, n=n, n_src=max(2, n // 50), n_tag=3, p_unmatched=0.2)
+    g, _ = gpu_batches(ORD, 1, n, n, single_batch(q))
+    o, _ = oracle_batches(ORD, 1, single_batch(q))
+    assert_exact(g, o)
+
+
+def test_ordered_wide_keys_and_wildcard_values():
+    rng = np.random.default_rng(1)
+    n = 20000
+    src = rng.integers(0, 1 << 32, n, dtype=np.uint64)
+    tag = rng.integers(0, 1 << 16, n, dtype=np.uint64)
+    comm = rng.integers(0, 1 << 16, n, dtype=np.uint64)
+    src[::7] = synth.ANY_SOURCE
+    tag[::5] = synth.ANY_TAG
+    rh = synth.pack(src, tag, comm)
+    rh[::3] = rh[0]
+    mh = rh[rng.permutation(n)]
+    b = [(rh, None, np.array([0, n]), mh, None, np.array([0, n]))]
+    g, _ = gpu_batches(ORD, 1, n, n, b)
+    o, _ = oracle_batches(ORD, 1, b)
+    assert_exact(g, o)
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_ordered_multibatch(seed):
+    rng = np.random.default_rng(seed)
+    q = synth.nowild_pairs(seed + 3, n=30000, n_src=300, n_tag=4, p_unmatched=0.3)
+    batches = split_batches(q, 3, rng)
+    g, _ = gpu_batches(ORD, 1, 60000, 60000, batches)
+    o, _ = oracle_batches(ORD, 1, batches)
+    assert_exact(g, o)
+
+
+def test_ordered_all_same_key():
+    n = 10000
+    rh = synth.pack(np.full(n, 4), np.full(n, 2))
+    mh = synth.pack(np.full(n - 17, 4), np.full(n - 17, 2))
+    b = [(rh, None, np.array([0, n]), mh, None, np.array([0, n - 17]))]
+    g, _ = gpu_batches(ORD, 1, n, n, b)
+    o, _ = oracle_batches(ORD, 1, b)
+    assert_exact(g, o)
+
+
+@pytest.mark.slow
+def test_ordered_config2_full():
+    q = synth.nowild_pairs()
+    n = len(q.recv_hdr)
+    g, _ = gpu_batches(ORD, 1, n, n, single_batch(q))
+    mr, _ = oracle.nowild_ordered(q.recv_hdr, q.msg_hdr)
+    grc, gmc, cnt = g[0]
+    assert np.array_equal(grc, np.arange(n))
+    assert np.array_equal(gmc, mr), "mismatches: %d" % int((gmc != mr).sum())
+
+
+@pytest.mark.parametrize("seed", range(5))
+@pytest.mark.parametrize("n", [1, 100, 5000, 70000])
+def test_unordered_random(seed, n):
+    q = synth.nowild_pairs(seed, n=n, n_src=max(2, n // 20), n_tag=3, p_unmatched=0.2)
+    g, _ = gpu_batches(UNO, 1, n, n, single_batch(q))
+    grc, gmc, cnt = g[0]
+    assert np.array_equal(grc, np.arange(n))
+    o, _ = oracle_batches(UNO, 1, single_batch(q))
+    # per-tuple counts are unique: compare them with the oracle's result
+    orc, omc = o[0]
+    om = omc >= 0
+    keys, counts = np.unique(q.recv_hdr[orc[om]], return_counts=True)
+    check_unordered(q.recv_hdr, q.msg_hdr, grc, gmc, dict(zip(keys.tolist(), counts.tolist())))
+    assert check_min(q) == int(cnt[1])
+
+
+def check_min(q):
+    return sum(per_key_min(q.recv_hdr, q.msg_hdr).values())
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_unordered_multibatch(seed):
+    rng = np.random.default_rng(seed)
+    q = synth.nowild_pairs(seed + 7, n=20000, n_src=200, n_tag=3, p_unmatched=0.3)
+    batches = split_batches(q, 3, rng)
+    g, _ = gpu_batches(UNO, 1, 40000, 40000, batches)
+    # across all batches: every pair has equal tuples, every element used once,
+    # and the total per tuple is min(#recv, #msg) of the whole input
+    rc = np.concatenate([x[0] for x in g])
+    mc = np.concatenate([x[1] for x in g])
+    m = mc >= 0
+    assert len(np.unique(rc[m])) == m.sum() and len(np.unique(mc[m])) == m.sum()
+    assert np.array_equal(q.recv_hdr[rc[m]], q.msg_hdr[mc[m]])
+    assert int(m.sum()) == check_min(q)
+
+
+@pytest.mark.slow
+def test_unordered_config3_per_gpu():
+    q = synth.nowild_pairs(3, n=1 << 25, n_src=1 << 20, n_tag=1 << 12)
+    n = len(q.recv_hdr)
+    g, _ = gpu_batches(UNO, 1, n, n, single_batch(q))
+    grc, gmc, cnt = g[0]
+    m = gmc >= 0
+    assert np.array_equal(q.recv_hdr[grc[m]], q.msg_hdr[gmc[m]])
+    assert len(np.unique(gmc[m])) == int(m.sum())
+    keys, mins = per_key_min_np(q.recv_hdr, q.msg_hdr)
+    assert int(m.sum()) == int(mins.sum()) == int(cnt[1])
+
+
+# ------------------------------------------------------------------- route
+
+
+@pytest.mark.parametrize("world,by", [(1, 0), (2, 0), (8, 0), (5, 1), (256, 0)])
+def test_route_stable_partition(world, by):
+    import torch
+    from paper_conf_ipps_klenkfed17_b200 import route
+    rng = np.random.default_rng(world)
+    n = 30011
+    if by == 0:
+        a = synth.pack(rng.integers(0, 1000, n), rng.integers(0, 50, n))
+        h = np.array([oracle.jenkins32((int(x) & 0xFFFFFFFF) ^ oracle.jenkins32(int(x) >> 32)) for x in a],
+                     dtype=np.uint64)
+        owner = (h * np.uint64(world)) >> np.uint64(32)
+    else:
+        owner = rng.integers(0, world, n).astype(np.uint64)
+        a = (owner << np.uint64(40)) | rng.integers(0, 1 << 40, n).astype(np.uint64)
+    b = rng.integers(0, 1 << 60, n)
+    da = torch.from_numpy(a.view(np.int64)).cuda()
+    db = torch.from_numpy(b).cuda()
+    oa = torch.empty_like(da)
+    ob = torch.empty_like(db)
+    counts = np.zeros(world, np.int64)
+    route(da, db, world, by, oa, ob, counts)
+    order = np.argsort(owner, kind="stable")
+    assert np.array_equal(counts, np.bincount(owner.astype(np.int64), minlength=world))
+    assert np.array_equal(oa.cpu().numpy().view(np.uint64), a[order])
+    assert np.array_equal(ob.cpu().numpy(), b[order])
