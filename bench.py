@@ -36,6 +36,7 @@ sys.path.insert(0, ROOT)
 
 METRIC = "matches/sec per semantics level (device-timed) at 1/2/4/8 B200; HBM GB/s"
 WORKLOADS = {
+    "mpi_matrix": "configs[1] on the compatibility-matrix kernel (MM_MPI_KERNEL_MATRIX)",
     "mpi": "configs[1]: MPI-compliant with wildcards, 4096 endpoints x 1024-deep recv/msg queues, "
            "proxy-app-shaped src/tag mix (10-30 peers, 1..4096 tags), 5% ANY_SOURCE",
     "ordered": "configs[2]: no wildcards, per-(src,tag) ordering kept: 16M recv/msg pairs via sort+rank pairing",
@@ -142,7 +143,7 @@ def to_dev(a):
 
 
 # --------------------------------------------------------------- our levels
-def bench_mpi(args, world, rank, peak):
+def bench_mpi(args, world, rank, peak, kernel=2, level="mpi"):
     import torch
 
     import paper_conf_ipps_klenkfed17_b200 as mm
@@ -157,7 +158,7 @@ def bench_mpi(args, world, rank, peak):
     orc = [torch.empty(n_r, dtype=torch.int64, device="cuda") for _ in range(ncopy)]
     omc = [torch.empty(n_r, dtype=torch.int64, device="cuda") for _ in range(ncopy)]
     cnt = [torch.zeros(2, dtype=torch.int64, device="cuda") for _ in range(ncopy)]
-    eng = mm.Engine(mm.MM_SEM_MPI, n_ep, depth, depth)
+    eng = mm.Engine(mm.MM_SEM_MPI, n_ep, depth, depth, mpi_kernel=kernel)
 
     def step(i):
         s = i % ncopy
@@ -174,10 +175,12 @@ def bench_mpi(args, world, rank, peak):
     # algorithmic bytes of the matcher kernel per launch: every header read
     # once, (recv cookie, msg cookie) written per receive, survivors compacted
     algo = 8 * (n_r + n_m) + 16 * n_r + 16 * resid
-    res.update(matches_per_step=matches, algo_bytes=algo, kernel="k_mpi_matrix", n_recv=n_r, n_msg=n_m)
-    res["e2e"] = bench_mpi_e2e(args, q, eng, world)
+    res.update(matches_per_step=matches, algo_bytes=algo, n_recv=n_r, n_msg=n_m,
+               kernel="k_mpi_fifo" if kernel == 2 else "k_mpi_matrix")
+    if level == "mpi":
+        res["e2e"] = bench_mpi_e2e(args, q, eng, world)
     eng.close()
-    return finish_level(res, world, peak, "mpi")
+    return finish_level(res, world, peak, level)
 
 
 def bench_mpi_e2e(args, q, eng, world):
@@ -371,7 +374,7 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--levels", default="mpi,ordered,unordered")
+    ap.add_argument("--levels", default="mpi,mpi_matrix,ordered,unordered")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
@@ -391,6 +394,8 @@ def main():
     wanted = args.levels.split(",")
     if "mpi" in wanted:
         levels["mpi"] = bench_mpi(args, world, rank, peak)
+    if "mpi_matrix" in wanted:
+        levels["mpi_matrix"] = bench_mpi(args, world, rank, peak, kernel=1, level="mpi_matrix")
     for lv in ("ordered", "unordered"):
         if lv in wanted:
             levels[lv] = bench_flat(args, world, rank, peak, lv)

@@ -165,18 +165,40 @@ int mm_destroy(mm_engine *e);
  * mm_route -- stable partition of n (a, b) pairs by owner rank, used to shard
  * the no-wildcard levels' tuple key space over `world` GPUs (DESIGN.md §1
  * row A6) and to return results to their origin.
- *   by == 0: owner = hash(a) * world >> 32, a = header word (key partition);
- *   by == 1: owner = a >> 40, a = cookie carrying the origin rank in bits
+ *   by == 0: owner = (hash(a) * world) >> 32, a = header word (key partition;
+ *            hash = the Jenkins fold of DESIGN.md reading R7);
+ *   by == 1: owner = a >> 40, a = a cookie carrying its origin rank in bits
  *            40..63 (result return trip).
- *   a, b        n inputs (device).  b may be NULL: the local index is used.
+ *   a           n inputs (device).
+ *   b           n inputs (device), or NULL: b[k] = cookie_base + k.  The
+ *               sharded path passes cookie_base = (rank << 40) | sequence, so
+ *               each cookie names its origin rank and a running local index.
+ *   cookie_base see b (>= 0).
  *   out_a/out_b n outputs (device), grouped by owner 0..world-1, each group in
  *               input order.
  *   counts      int64[world] (device or host) elements per owner.
- *   world       1..1024.
+ *   world       1..256.
  *   stream      cudaStream_t as void*.
+ * Synchronises the stream only when `counts` is host memory.
  */
 int mm_route(const uint64_t *a, const int64_t *b, int64_t n, int32_t world, int32_t by,
-             uint64_t *out_a, int64_t *out_b, int64_t *counts, void *stream);
+             int64_t cookie_base, uint64_t *out_a, int64_t *out_b, int64_t *counts, void *stream);
+
+/*
+ * mm_set_option -- engine tuning knobs (host-side, takes effect at the next
+ * mm_match_batch).
+ *   MM_OPT_MPI_KERNEL: which kernel implements the MPI level --
+ *     MM_MPI_KERNEL_FIFO (default, MM_MPI_KERNEL_AUTO): per-tuple FIFO lists,
+ *       exact receives resolved by prefix counts, wildcards by a warp search
+ *       (DESIGN.md §2.3, §7.2);
+ *     MM_MPI_KERNEL_MATRIX: the paper's compatibility-matrix scan/reduce
+ *       (§V.A Alg. 1-2) re-designed per warp.
+ *   Both produce identical results.  Returns MM_ERR_ARG for unknown options
+ *   or values.
+ */
+enum { MM_OPT_MPI_KERNEL = 1 };
+enum { MM_MPI_KERNEL_AUTO = 0, MM_MPI_KERNEL_MATRIX = 1, MM_MPI_KERNEL_FIFO = 2 };
+int mm_set_option(mm_engine *e, int32_t option, int64_t value);
 
 /* mm_strerror -- static description of an MM_* code. */
 const char *mm_strerror(int code);

@@ -22,6 +22,9 @@ MM_ERR_CAPACITY = 3
 MM_ERR_NOMEM = 4
 MM_ERR_STATE = 5
 
+MM_OPT_MPI_KERNEL = 1
+MM_MPI_KERNEL_AUTO, MM_MPI_KERNEL_MATRIX, MM_MPI_KERNEL_FIFO = 0, 1, 2
+
 MM_NO_MATCH = -1
 MM_ANY_SOURCE = 0xFFFFFFFF
 MM_ANY_TAG = 0xFFFF
@@ -42,7 +45,8 @@ SIGNATURES = {
     "mm_reset": (ctypes.c_int, [_P]),
     "mm_query": (ctypes.c_int, [_P, _P]),
     "mm_destroy": (ctypes.c_int, [_P]),
-    "mm_route": (ctypes.c_int, [_P, _P, _I64, _I32, _I32, _P, _P, _P, _P]),
+    "mm_route": (ctypes.c_int, [_P, _P, _I64, _I32, _I32, _I64, _P, _P, _P, _P]),
+    "mm_set_option": (ctypes.c_int, [_P, _I32, _I64]),
     "mm_strerror": (ctypes.c_char_p, [ctypes.c_int]),
     "mm_version": (ctypes.c_char_p, []),
 }

@@ -397,9 +397,10 @@ struct MoveRoute {
   const int64_t* b;
   uint64_t* oa;
   int64_t* ob;
+  int64_t base;
   __device__ __forceinline__ void operator()(int64_t k, int64_t dst) const {
     oa[dst] = a[k];
-    ob[dst] = b ? b[k] : k;
+    ob[dst] = b ? b[k] : (base + k);
   }
 };
 __global__ void k_route_counts(const uint32_t* hist, int64_t ntiles, int world, int64_t n, int64_t* counts) {
@@ -411,10 +412,10 @@ __global__ void k_route_counts(const uint32_t* hist, int64_t ntiles, int world, 
   }
 }
 
-cudaError_t run_route(const uint64_t* a, const int64_t* b, int64_t n, int world, int by, uint64_t* out_a,
+cudaError_t run_route(const uint64_t* a, const int64_t* b, int64_t n, int world, int by, int64_t cookie_base, uint64_t* out_a,
                       int64_t* out_b, int64_t* counts, uint32_t* part, cudaStream_t st) {
   if (n == 0) return cudaMemsetAsync(counts, 0, sizeof(int64_t) * world, st);
-  cudaError_t err = partition_stable(OwnerOf{a, world, by}, MoveRoute{a, b, out_a, out_b}, n, world, part, st);
+  cudaError_t err = partition_stable(OwnerOf{a, world, by}, MoveRoute{a, b, out_a, out_b, cookie_base}, n, world, part, st);
   if (err != cudaSuccess) return err;
   int64_t nt = (n + kPartTile - 1) / kPartTile;
   count_launch();

@@ -139,6 +139,9 @@ struct mm_engine {
   DBuf out_rc_stage, out_mc_stage;
   // MPI
   int64_t msg_slots = 0, warp_words = 0;
+  int mpi_kernel = MM_MPI_KERNEL_FIFO;
+  FifoLayout fifo{};
+  DBuf fifo_ws;
   // single-endpoint levels
   DBuf rflag, mflag, scan;
   DBuf skey[2], sval[2], rid, run_start, run_rc, part;
@@ -224,7 +227,7 @@ int mm_destroy(mm_engine* e) {
   DBuf* bufs[] = {&e->out_off, &e->counts_dev, &e->nmatched, &e->err, &e->info, &e->out_rc_stage,
                   &e->out_mc_stage, &e->rflag, &e->mflag, &e->scan, &e->skey[0], &e->skey[1],
                   &e->sval[0], &e->sval[1], &e->rid, &e->run_start, &e->run_rc, &e->part,
-                  &e->owner, &e->rcnt, &e->mcnt, &e->tkey, &e->tval};
+                  &e->owner, &e->rcnt, &e->mcnt, &e->tkey, &e->tval, &e->fifo_ws};
   for (DBuf* b : bufs) release(*b);
   delete e;
   return MM_OK;
@@ -263,6 +266,9 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
   if (ok && semantics == MM_SEM_MPI) {
     e->msg_slots = (e->mcap + 63) / 64 * 64;
     e->warp_words = (e->msg_slots + e->msg_slots / 64 + 3) / 4 * 4;  // headers + availability bits, 32 B aligned
+    e->fifo = fifo_layout(e->rcap, e->mcap);
+    if (!e->fifo.in_smem)
+      ok = ensure(e->fifo_ws, (size_t)fifo_grid(e->fifo, n_endpoints) * (size_t)e->fifo.total) == cudaSuccess;
   }
   if (ok && semantics != MM_SEM_MPI) {
     const int64_t n = e->rcap + e->mcap;
@@ -427,7 +433,10 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
   a.n_matched = (unsigned long long*)e->nmatched.p;
   a.err = (uint32_t*)e->err.p;
   e->timer.begin(e->st);
-  CK(launch_mpi_matrix(a, e->st));
+  if (e->mpi_kernel == MM_MPI_KERNEL_MATRIX)
+    CK(launch_mpi_matrix(a, e->st));
+  else
+    CK(launch_mpi_fifo(a, e->fifo, (uint8_t*)e->fifo_ws.p, e->st));
   e->timer.end(e->st);
   CK(launch_finalize((const int64_t*)e->out_off.p + e->n_ep, 0, (const unsigned long long*)e->nmatched.p,
                      (int64_t*)e->counts_dev.p, e->st));
@@ -532,6 +541,17 @@ int mm_match_batch(mm_engine* e, int64_t* out_recv_cookie, int64_t* out_msg_cook
   return match_flat(e, out_recv_cookie, out_msg_cookie, out_capacity, counts);
 }
 
+int mm_set_option(mm_engine* e, int32_t option, int64_t value) {
+  if (!e) return MM_ERR_ARG;
+  if (option == MM_OPT_MPI_KERNEL) {
+    if (value == MM_MPI_KERNEL_AUTO) value = MM_MPI_KERNEL_FIFO;
+    if (value != MM_MPI_KERNEL_MATRIX && value != MM_MPI_KERNEL_FIFO) return MM_ERR_ARG;
+    e->mpi_kernel = (int)value;
+    return MM_OK;
+  }
+  return MM_ERR_ARG;
+}
+
 int mm_query(mm_engine* e, int64_t* vals) {
   if (!e || !vals) return MM_ERR_ARG;
   CK(cudaStreamSynchronize(e->st));
@@ -563,9 +583,9 @@ int mm_query(mm_engine* e, int64_t* vals) {
   return err ? MM_ERR_CAPACITY : MM_OK;
 }
 
-int mm_route(const uint64_t* a, const int64_t* b, int64_t n, int32_t world, int32_t by, uint64_t* out_a,
-             int64_t* out_b, int64_t* counts, void* stream) {
-  if (n < 0 || world < 1 || world > 256 || (by != 0 && by != 1)) return MM_ERR_ARG;
+int mm_route(const uint64_t* a, const int64_t* b, int64_t n, int32_t world, int32_t by, int64_t cookie_base,
+             uint64_t* out_a, int64_t* out_b, int64_t* counts, void* stream) {
+  if (n < 0 || world < 1 || world > 256 || (by != 0 && by != 1) || cookie_base < 0) return MM_ERR_ARG;
   if (n > 0 && (!a || !out_a || !out_b)) return MM_ERR_ARG;
   if (!counts) return MM_ERR_ARG;
   if (n >= ((int64_t)1 << 32)) return MM_ERR_ARG;
@@ -577,7 +597,7 @@ int mm_route(const uint64_t* a, const int64_t* b, int64_t n, int32_t world, int3
   void* dcounts = nullptr;
   CK(cudaMallocAsync(&part, (size_t)partition_scratch_elems(n > 0 ? n : 1) * 4, st));
   CK(cudaMallocAsync(&dcounts, (size_t)world * 8, st));
-  cudaError_t err = run_route(a, b, n, world, by, out_a, out_b, (int64_t*)dcounts, (uint32_t*)part, st);
+  cudaError_t err = run_route(a, b, n, world, by, cookie_base, out_a, out_b, (int64_t*)dcounts, (uint32_t*)part, st);
   if (err == cudaSuccess)
     err = cudaMemcpyAsync(counts, dcounts, (size_t)world * 8,
                           counts_host ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice, st);

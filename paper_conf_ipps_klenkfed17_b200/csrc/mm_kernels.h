@@ -24,6 +24,18 @@ struct MpiArgs {
   uint32_t* err;
 };
 
+// Key-FIFO engine workspace (byte offsets inside one CTA's workspace).
+constexpr int64_t kFifoSmemMax = 100 * 1024;
+struct FifoLayout {
+  int64_t msgs, table, slot_id, key_owner, key_cnt, key_start, key_e, key_c, msg_key, by_key, recv_key, matched;
+  int64_t total;
+  uint32_t H;
+  bool in_smem;
+};
+FifoLayout fifo_layout(int64_t rcap, int64_t mcap);
+int fifo_grid(const FifoLayout& L, int n_ep);
+cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws, cudaStream_t st);
+
 cudaError_t launch_out_offsets(const Side& R, int n_ep, int64_t* out_off, int64_t out_cap, uint32_t* err,
                                cudaStream_t st);
 cudaError_t launch_mpi_matrix(const MpiArgs& a, cudaStream_t st);
@@ -80,7 +92,7 @@ cudaError_t run_compact(const Side& S, int64_t resid, int64_t n, const uint8_t* 
                         int32_t* q_len, uint32_t* scan, cudaStream_t st);
 
 // mm_route
-cudaError_t run_route(const uint64_t* a, const int64_t* b, int64_t n, int world, int by, uint64_t* out_a,
+cudaError_t run_route(const uint64_t* a, const int64_t* b, int64_t n, int world, int by, int64_t cookie_base, uint64_t* out_a,
                       int64_t* out_b, int64_t* counts, uint32_t* part, cudaStream_t st);
 
 // counts[] = {n_out, n_matched} from device state

@@ -70,7 +70,8 @@ def current_stream_handle(device=None):
 class Engine:
     """Owns one mm_engine (see include/mm.h for the semantics of each call)."""
 
-    def __init__(self, semantics, n_endpoints=1, recv_capacity=1024, msg_capacity=1024, stream=None):
+    def __init__(self, semantics, n_endpoints=1, recv_capacity=1024, msg_capacity=1024, stream=None,
+                 mpi_kernel=None):
         L = _lib.load()
         self._L = L
         self.semantics = semantics
@@ -86,6 +87,11 @@ class Engine:
         check(L.mm_create(ctypes.byref(h), semantics, n_endpoints, recv_capacity, msg_capacity, stream), "mm_create")
         self._h = h
         self._keep = []  # device buffers referenced by pending batches
+        if mpi_kernel is not None:
+            self.set_option(_lib.MM_OPT_MPI_KERNEL, mpi_kernel)
+
+    def set_option(self, option, value):
+        check(self._L.mm_set_option(self._h, option, value), "mm_set_option")
 
     def _post(self, fn, name, hdr, cookie, ep_offsets):
         hdr = _as_u64(hdr)
@@ -137,11 +143,11 @@ class Engine:
         self.close()
 
 
-def route(a, b, world, by, out_a, out_b, counts, stream=None):
+def route(a, b, world, by, out_a, out_b, counts, stream=None, cookie_base=0):
     """mm_route: stable partition of (a, b) by owner rank (device tensors)."""
     L = _lib.load()
     if stream is None:
         stream = current_stream_handle()
-    check(L.mm_route(_ptr(a), _ptr(b), _len(a), world, by, _ptr(out_a), _ptr(out_b), _ptr(counts), stream),
-          "mm_route")
+    check(L.mm_route(_ptr(a), _ptr(b), _len(a), world, by, cookie_base, _ptr(out_a), _ptr(out_b), _ptr(counts),
+                     stream), "mm_route")
     return out_a, out_b, counts

@@ -62,7 +62,7 @@ def test_argument_errors_without_device():
     assert L.mm_post_recvs(None, None, None, None, 0) == _lib.MM_ERR_ARG
     assert L.mm_match_batch(None, None, None, 0, None) == _lib.MM_ERR_ARG
     assert L.mm_destroy(None) == _lib.MM_OK
-    assert L.mm_route(None, None, 0, 0, 0, None, None, None, None) == _lib.MM_ERR_ARG
+    assert L.mm_route(None, None, 0, 0, 0, 0, None, None, None, None) == _lib.MM_ERR_ARG
 
 
 @pytest.mark.skipif(gpu_available(), reason="checks the no-device path")

@@ -16,6 +16,7 @@ from _util import (check_unordered, gpu_batches, oracle_batches, per_key_min, pe
 pytestmark = pytest.mark.gpu
 
 MPI, ORD, UNO = oracle.SEM_MPI, oracle.SEM_NOWILD_ORDERED, oracle.SEM_NOWILD_UNORDERED
+KERNELS = pytest.mark.parametrize("kern", [1, 2], ids=["matrix", "fifo"])  # MM_MPI_KERNEL_*
 
 
 def assert_exact(g, o):
@@ -29,47 +30,52 @@ def assert_exact(g, o):
         assert int(cnt[1]) == int((omc >= 0).sum())
 
 
-def test_mpi_config0():
+@KERNELS
+def test_mpi_config0(kern):
     q = synth.mpi_small(0)
-    g, _ = gpu_batches(MPI, 1, 64, 64, single_batch(q))
+    g, _ = gpu_batches(MPI, 1, 64, 64, single_batch(q), mpi_kernel=kern)
     o, _ = oracle_batches(MPI, 1, single_batch(q))
     assert_exact(g, o)
 
 
 @pytest.mark.parametrize("seed", range(6))
 @pytest.mark.parametrize("depth", [1, 31, 33, 200, 1024])
-def test_mpi_ragged_endpoints(seed, depth):
+@KERNELS
+def test_mpi_ragged_endpoints(seed, depth, kern):
     q = synth.mpi_endpoints(seed, n_ep=37, depth_r=depth, n_src=5, n_tag=4, p_any_src=0.3, p_any_tag=0.3,
                             n_comm=2, ragged=True, p_unmatched=0.2)
-    g, qs = gpu_batches(MPI, q.n_endpoints, depth, depth, single_batch(q))
+    g, qs = gpu_batches(MPI, q.n_endpoints, depth, depth, single_batch(q), mpi_kernel=kern)
     o, _ = oracle_batches(MPI, q.n_endpoints, single_batch(q))
     assert_exact(g, o)
     assert qs["error"] == 0
 
 
 @pytest.mark.parametrize("seed", range(4))
-def test_mpi_multibatch_residuals(seed):
+@KERNELS
+def test_mpi_multibatch_residuals(seed, kern):
     rng = np.random.default_rng(seed)
     q = synth.mpi_endpoints(seed + 10, n_ep=50, depth_r=150, n_src=4, n_tag=3, p_any_src=0.25, p_any_tag=0.25,
                             ragged=True, p_unmatched=0.3)
     batches = split_batches(q, 4, rng)
-    g, qs = gpu_batches(MPI, q.n_endpoints, 600, 600, batches)
+    g, qs = gpu_batches(MPI, q.n_endpoints, 600, 600, batches, mpi_kernel=kern)
     o, oe = oracle_batches(MPI, q.n_endpoints, batches)
     assert_exact(g, o)
     rr, rm = oe.residual_depths()
     assert qs["resid_recv"] == sum(rr) and qs["resid_msg"] == sum(rm)
 
 
-def test_mpi_host_buffers_equal_device():
+@KERNELS
+def test_mpi_host_buffers_equal_device(kern):
     q = synth.mpi_endpoints(5, n_ep=64, depth_r=128, ragged=True, p_unmatched=0.1)
-    gd, _ = gpu_batches(MPI, q.n_endpoints, 128, 128, single_batch(q))
-    gh, _ = gpu_batches(MPI, q.n_endpoints, 128, 128, single_batch(q), host=True)
+    gd, _ = gpu_batches(MPI, q.n_endpoints, 128, 128, single_batch(q), mpi_kernel=kern)
+    gh, _ = gpu_batches(MPI, q.n_endpoints, 128, 128, single_batch(q), host=True, mpi_kernel=kern)
     o, _ = oracle_batches(MPI, q.n_endpoints, single_batch(q))
     assert_exact(gd, o)
     assert_exact(gh, o)
 
 
-def test_mpi_user_cookies_and_two_posts():
+@KERNELS
+def test_mpi_user_cookies_and_two_posts(kern):
     """Cookies are carried through; a second post before a match is queued."""
     q = synth.mpi_endpoints(6, n_ep=8, depth_r=64, p_unmatched=0.1)
     rng = np.random.default_rng(0)
@@ -89,7 +95,7 @@ def test_mpi_user_cookies_and_two_posts():
     import torch
     from _util import to_dev
     from paper_conf_ipps_klenkfed17_b200 import Engine
-    eng = Engine(MPI, 8, 64, 64)
+    eng = Engine(MPI, 8, 64, 64, mpi_kernel=kern)
     eng.post_recvs(to_dev(ra[0]), to_dev(ra[1]), to_dev(ra[2]))
     eng.push_msgs(to_dev(ma[0]), to_dev(ma[1]), to_dev(ma[2]))
     eng.post_recvs(to_dev(rb[0]), to_dev(rb[1]), to_dev(rb[2]))
@@ -110,41 +116,45 @@ def test_mpi_user_cookies_and_two_posts():
     eng.close()
 
 
-def test_mpi_empty_and_degenerate():
+@KERNELS
+def test_mpi_empty_and_degenerate(kern):
     # no receives at all, no messages at all, both empty
     for nr, nm in [(0, 10), (10, 0), (0, 0)]:
         rh = synth.pack(np.arange(nr) % 3, np.zeros(nr, int))
         mh = synth.pack(np.arange(nm) % 3, np.zeros(nm, int))
         b = [(rh, None, np.array([0, nr]), mh, None, np.array([0, nm]))]
-        g, _ = gpu_batches(MPI, 1, 16, 16, b)
+        g, _ = gpu_batches(MPI, 1, 16, 16, b, mpi_kernel=kern)
         o, _ = oracle_batches(MPI, 1, b)
         assert_exact(g, o)
     # all (ANY, ANY) receives against many senders
     rh = synth.pack(np.full(100, synth.ANY_SOURCE), np.full(100, synth.ANY_TAG))
     mh = synth.pack(np.arange(90) % 7, np.arange(90) % 5)
     b = [(rh, None, np.array([0, 100]), mh, None, np.array([0, 90]))]
-    g, _ = gpu_batches(MPI, 1, 128, 128, b)
+    g, _ = gpu_batches(MPI, 1, 128, 128, b, mpi_kernel=kern)
     o, _ = oracle_batches(MPI, 1, b)
     assert_exact(g, o)
 
 
-def test_mpi_capacity_overflow_is_flagged():
+@KERNELS
+def test_mpi_capacity_overflow_is_flagged(kern):
     q = synth.mpi_endpoints(3, n_ep=4, depth_r=40)
-    g, qs = gpu_batches(MPI, 4, 32, 32, single_batch(q), out_cap=4 * 40)
+    g, qs = gpu_batches(MPI, 4, 32, 32, single_batch(q), out_cap=4 * 40, mpi_kernel=kern)
     assert qs["error"] != 0 and qs["rc"] == 3
 
 
-def test_mpi_config4_worst_chain():
+@KERNELS
+def test_mpi_config4_worst_chain(kern):
     q = synth.worst_chain()
-    g, _ = gpu_batches(MPI, 1, 16384, 16384, single_batch(q))
+    g, _ = gpu_batches(MPI, 1, 16384, 16384, single_batch(q), mpi_kernel=kern)
     o, _ = oracle_batches(MPI, 1, single_batch(q))
     assert_exact(g, o)
 
 
 @pytest.mark.slow
-def test_mpi_config1_full():
+@KERNELS
+def test_mpi_config1_full(kern):
     q = synth.proxy_endpoints()
-    g, qs = gpu_batches(MPI, q.n_endpoints, 1024, 1024, single_batch(q))
+    g, qs = gpu_batches(MPI, q.n_endpoints, 1024, 1024, single_batch(q), mpi_kernel=kern)
     mr, _ = oracle.mpi_endpoints(q)
     grc, gmc, cnt = g[0]
     assert np.array_equal(grc, np.arange(len(q.recv_hdr)))
@@ -285,6 +295,10 @@ def test_route_stable_partition(world, by):
     ob = torch.empty_like(db)
     counts = np.zeros(world, np.int64)
     route(da, db, world, by, oa, ob, counts)
+    # b == NULL: generated cookies cookie_base + k
+    oa2, ob2 = torch.empty_like(da), torch.empty_like(db)
+    route(da, None, world, by, oa2, ob2, counts, cookie_base=(3 << 40) + 7)
+    assert np.array_equal(ob2.cpu().numpy(), (3 << 40) + 7 + np.argsort(owner, kind="stable"))
     order = np.argsort(owner, kind="stable")
     assert np.array_equal(counts, np.bincount(owner.astype(np.int64), minlength=world))
     assert np.array_equal(oa.cpu().numpy().view(np.uint64), a[order])
