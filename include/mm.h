@@ -96,7 +96,7 @@ typedef struct mm_engine mm_engine; /* opaque, owned by the library */
  *                   The no-wildcard levels require n_endpoints == 1 (the
  *                   comm field still separates communicators).
  *   recv_capacity   max receives in one endpoint's batch snapshot (residual
- *                   PRQ + newly posted), > 0.
+ *                   PRQ + newly posted), > 0; <= MM_MPI_MAX_RECVS under MM_SEM_MPI.
  *   msg_capacity    max messages in one endpoint's snapshot, > 0.  Under
  *                   MM_SEM_MPI one endpoint's messages are staged on chip, so
  *                   msg_capacity <= MM_MPI_MAX_MSGS.
@@ -105,6 +105,7 @@ typedef struct mm_engine mm_engine; /* opaque, owned by the library */
  *   out             receives the engine handle (owned; free with mm_destroy).
  */
 #define MM_MPI_MAX_MSGS 24576
+#define MM_MPI_MAX_RECVS 65534
 int mm_create(mm_engine **out, int32_t semantics, int32_t n_endpoints,
               int64_t recv_capacity, int64_t msg_capacity, void *stream);
 

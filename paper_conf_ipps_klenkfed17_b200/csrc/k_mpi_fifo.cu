@@ -1,77 +1,119 @@
-// k_mpi_fifo.cu -- full MPI semantics, key-FIFO engine (rows A2-A3, DESIGN.md §1, §7.2).
+// k_mpi_fifo.cu -- full MPI semantics, key-FIFO engine (rows A2-A3, DESIGN.md §1, §2.3, §7.2).
 //
-// Observation: under "each receive, in posting order, takes
-// the earliest-arrived unmatched message it admits", every receive consumes
-// the HEAD of one per-tuple FIFO -- an exact receive the head of its own
-// tuple's list, a wildcard receive the earliest head among the tuples it
-// admits.  So the state of an endpoint is one consumption counter per tuple,
-// and an exact receive of tuple k at posting position i takes
-//     list_k[ e_k(i) + c_k(i) ]   (if < n_k, else nothing),
-// with e_k(i) the exact receives of k before i (a prefix count) and c_k(i)
-// the wildcard receives before i that took from k (the claims earlier
-// wildcards retired from the list).  Only wildcard receives need a search.
+// Under "each receive, in posting order, takes the earliest-arrived unmatched
+// message it admits" every receive consumes the HEAD of one per-tuple FIFO:
+// an exact receive the head of its own tuple's list, a wildcard receive the
+// earliest head among the tuples it admits.  Hence an exact
+// receive of tuple k at posting position i takes
+//     list_k[ e_i + c_k(i) ]            (nothing if >= n_k)
+// with e_i its rank among the exact receives of k (a prefix count) and c_k(i)
+// the number of wildcard receives before i that took from k -- the claims
+// earlier receives retired from the list.  Only wildcards need a search, and
+// only they are processed sequentially.
 //
-// Per endpoint (one CTA, workspace in shared memory, or in an L2-resident
-// global slice for deep queues):
-//  1. stage message headers (16-byte vector loads) and insert them into an
-//     open-addressing hash table (16-bit CAS); dense tuple ids by block scan;
-//     per-tuple counts and starts by block scan; one warp places messages into
-//     their tuple lists in arrival order (match_any ranks), while the other
-//     warps classify receives (exact tuple id / wildcard / absent tuple);
-//  2. one warp sweeps the receives in posting order, 32 at a time: exact
-//     receives between two wildcards resolve together (match_any gives the
-//     rank among equal tuples, the per-tuple counters give the prefix); a
-//     wildcard receive makes the warp scan the tuples, test admissibility with
-//     one masked XOR, read each admitted tuple's head and take the minimum
-//     arrival index (redux.sync.min), retiring the claim by bumping c_k;
-//  3. results, and the in-place compaction of both queues, are written with
-//     ballot/popc prefix ranks.
-// Results equal the definition exactly (no ties: arrival indices are unique).
+// Per endpoint (one CTA; workspace in shared memory, or an L2-resident global
+// slice for deep queues):
+//  P1 stage message and receive headers (16-byte loads);
+//  P2 insert message tuples into an open-addressing hash table (16-bit CAS);
+//  P3 dense tuple ids (block scan over slots);
+//  P4 classify receives (tuple id / wildcard / tuple absent), count messages
+//     and exact receives per tuple;
+//  P5 block scans: tuple list starts for both sides, ordered wildcard list;
+//  P6 warp 0 places messages, warp 1 places exact receives into their tuple
+//     lists in order (match_any ranks) -- giving every exact receive its e_i;
+//  P7 warp 0 walks the wildcards in posting order: lanes test admissibility of
+//     tuples with one masked XOR, read each admitted tuple's head
+//     (e_k(w) from a per-tuple cursor over that tuple's exact receives, plus
+//     c_k) and redux.sync.min picks the earliest arrival; the winner tuple's
+//     c_k is bumped and the claim logged (wlog_k);
+//  P8 all threads resolve exact receives: c_k(i) = claims in wlog_k before i;
+//     results are written coalesced and unmatched receives compacted in order
+//     (block-scan ranks);
+//  P9 unmatched messages compacted in arrival order.
+// Exact by construction: no ties (arrival indices are unique).
 #include "mm_kernels.h"
 
 namespace mm {
 
-constexpr uint32_t kRecvWild = 0xFFFFFFFEu;
-constexpr uint32_t kRecvNone = 0xFFFFFFFFu;
-constexpr uint16_t kSlotEmpty = 0xFFFFu;
+constexpr uint16_t kWild = 0xFFFEu;
+constexpr uint16_t kNone = 0xFFFFu;
+constexpr uint16_t kEmpty16 = 0xFFFFu;
 
 struct FifoWs {
-  uint64_t* msgs;      // [mcap] message headers
-  uint16_t* table;     // [H] slot -> representative message (kSlotEmpty)
-  uint16_t* slot_id;   // [H] slot -> dense tuple id
-  uint16_t* key_owner; // [mcap] tuple id -> representative message
-  uint32_t* key_cnt;   // [mcap] n_k
-  uint32_t* key_start; // [mcap] start of tuple k's list in by_key
-  uint32_t* key_e;     // [mcap] exact receives of k seen by the sweep
-  uint32_t* key_c;     // [mcap] wildcard receives that took from k
-  uint32_t* msg_key;   // [mcap] message -> slot, then -> tuple id
-  uint16_t* by_key;    // [mcap] message indices grouped by tuple, arrival order
-  uint32_t* recv_key;  // [rcap] receive -> tuple id | kRecvWild | kRecvNone
-  uint32_t* matched;   // [mcap/32] message matched bits
+  uint64_t* msgs;       // [mcap] staged message headers
+  uint64_t* recvs;      // [rcap] staged receive headers
+  uint64_t* keyhdr;     // [mcap] tuple id -> header
+  uint16_t* table;      // [H] slot -> representative message
+  uint16_t* slot_id;    // [H] slot -> dense tuple id
+  uint16_t* key_cnt;    // [mcap] messages of tuple k
+  uint16_t* key_start;  // [mcap] start of tuple k in by_key / wlog
+  uint16_t* key_rcnt;   // [mcap] exact receives of tuple k
+  uint16_t* key_rstart; // [mcap] start of tuple k in rby_key
+  uint16_t* key_c;      // [mcap] wildcard claims on tuple k
+  uint16_t* key_cur;    // [mcap] cursor over tuple k's exact receives
+  uint16_t* msg_key;    // [mcap] message -> slot, then tuple id
+  uint16_t* by_key;     // [mcap] messages grouped by tuple, arrival order
+  uint16_t* wlog;       // [mcap] per tuple: posting positions of the wildcards that claimed it
+  uint16_t* recv_key;   // [rcap] receive -> tuple id | kWild | kNone
+  uint16_t* recv_e;     // [rcap] rank among the exact receives of its tuple
+  uint16_t* rby_key;    // [rcap] exact receives grouped by tuple, posting order
+  uint16_t* recv_res;   // [rcap] wildcard results (message index | kNone)
+  uint16_t* wl;         // [rcap] wildcard positions in posting order
+  uint32_t* matched;    // [mcap/32] message matched bits
+  // wildcard groups (all wildcards of one type: tuples split by hdr & mask)
+  uint16_t* key_grp;    // [mcap] tuple -> group
+  uint16_t* g_cnt;      // [mcap] tuples per group (low) ...
+  uint16_t* g_start;    // [mcap] start of group g in g_keys
+  uint16_t* g_keys;     // [mcap] tuples grouped by group
+  uint16_t* gw_cnt;     // [mcap] wildcards per group
+  uint16_t* gw_start;   // [mcap] start of group g in gw_list
+  uint16_t* w_grp;      // [rcap] wildcard (index into wl) -> group | kNone
+  uint16_t* gw_list;    // [rcap] wildcards grouped by group, posting order
 };
 
 __device__ __forceinline__ FifoWs carve(uint8_t* base, const FifoLayout& L) {
   FifoWs w;
   w.msgs = reinterpret_cast<uint64_t*>(base + L.msgs);
+  w.recvs = reinterpret_cast<uint64_t*>(base + L.recvs);
+  w.keyhdr = reinterpret_cast<uint64_t*>(base + L.keyhdr);
   w.table = reinterpret_cast<uint16_t*>(base + L.table);
   w.slot_id = reinterpret_cast<uint16_t*>(base + L.slot_id);
-  w.key_owner = reinterpret_cast<uint16_t*>(base + L.key_owner);
-  w.key_cnt = reinterpret_cast<uint32_t*>(base + L.key_cnt);
-  w.key_start = reinterpret_cast<uint32_t*>(base + L.key_start);
-  w.key_e = reinterpret_cast<uint32_t*>(base + L.key_e);
-  w.key_c = reinterpret_cast<uint32_t*>(base + L.key_c);
-  w.msg_key = reinterpret_cast<uint32_t*>(base + L.msg_key);
+  w.key_cnt = reinterpret_cast<uint16_t*>(base + L.key_cnt);
+  w.key_start = reinterpret_cast<uint16_t*>(base + L.key_start);
+  w.key_rcnt = reinterpret_cast<uint16_t*>(base + L.key_rcnt);
+  w.key_rstart = reinterpret_cast<uint16_t*>(base + L.key_rstart);
+  w.key_c = reinterpret_cast<uint16_t*>(base + L.key_c);
+  w.key_cur = reinterpret_cast<uint16_t*>(base + L.key_cur);
+  w.msg_key = reinterpret_cast<uint16_t*>(base + L.msg_key);
   w.by_key = reinterpret_cast<uint16_t*>(base + L.by_key);
-  w.recv_key = reinterpret_cast<uint32_t*>(base + L.recv_key);
+  w.wlog = reinterpret_cast<uint16_t*>(base + L.wlog);
+  w.recv_key = reinterpret_cast<uint16_t*>(base + L.recv_key);
+  w.recv_e = reinterpret_cast<uint16_t*>(base + L.recv_e);
+  w.rby_key = reinterpret_cast<uint16_t*>(base + L.rby_key);
+  w.recv_res = reinterpret_cast<uint16_t*>(base + L.recv_res);
+  w.wl = reinterpret_cast<uint16_t*>(base + L.wl);
   w.matched = reinterpret_cast<uint32_t*>(base + L.matched);
+  w.key_grp = reinterpret_cast<uint16_t*>(base + L.key_grp);
+  w.g_cnt = reinterpret_cast<uint16_t*>(base + L.g_cnt);
+  w.g_start = reinterpret_cast<uint16_t*>(base + L.g_start);
+  w.g_keys = reinterpret_cast<uint16_t*>(base + L.g_keys);
+  w.gw_cnt = reinterpret_cast<uint16_t*>(base + L.gw_cnt);
+  w.gw_start = reinterpret_cast<uint16_t*>(base + L.gw_start);
+  w.w_grp = reinterpret_cast<uint16_t*>(base + L.w_grp);
+  w.gw_list = reinterpret_cast<uint16_t*>(base + L.gw_list);
   return w;
 }
 
-// 16-bit CAS on shared or global memory through the containing 32-bit word.
+// 16-bit CAS through the containing 32-bit word.
+// (pointer arithmetic, not integer casts, so shared-memory provenance survives
+// and the atomics compile to ATOMS)
+__device__ __forceinline__ uint32_t* word_of(uint16_t* p) {
+  return reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(p) - (reinterpret_cast<uintptr_t>(p) & 2));
+}
 __device__ __forceinline__ uint16_t cas16(uint16_t* p, uint16_t expect, uint16_t val) {
-  uint32_t* w = reinterpret_cast<uint32_t*>(reinterpret_cast<uintptr_t>(p) & ~uintptr_t(3));
+  uint32_t* w = word_of(p);
   const uint32_t sh = (reinterpret_cast<uintptr_t>(p) & 2) ? 16u : 0u;
-  uint32_t old = *reinterpret_cast<volatile uint32_t*>(w);
+  uint32_t old = *w;
   while (true) {
     const uint16_t cur = (uint16_t)(old >> sh);
     if (cur != expect) return cur;
@@ -82,19 +124,107 @@ __device__ __forceinline__ uint16_t cas16(uint16_t* p, uint16_t expect, uint16_t
   }
 }
 
-// Block-wide exclusive scan of per-thread chunk counts (all threads call).
-template <int NT>
-__device__ __forceinline__ uint32_t block_scan_u32(uint32_t v, uint32_t* sm, uint32_t* total) {
-  return block_excl_scan<uint32_t>(v, sm, total);
+// 16-bit counter increment through the containing 32-bit word (no carry out:
+// counts stay below 65536).
+__device__ __forceinline__ void inc16(uint16_t* p) {
+  atomicAdd(word_of(p), (reinterpret_cast<uintptr_t>(p) & 2) ? 0x10000u : 1u);
+}
+// Same, returning the previous 16-bit value.
+__device__ __forceinline__ uint32_t fetch_inc16(uint16_t* p) {
+  const bool hi = (reinterpret_cast<uintptr_t>(p) & 2) != 0;
+  const uint32_t old = atomicAdd(word_of(p), hi ? 0x10000u : 1u);
+  return hi ? (old >> 16) : (old & 0xFFFFu);
+}
+
+// One wildcard receive w (header r, mask msk) against candidate tuples
+// cand(0..nc) -- all admitted tuples are among them.  Lanes read each admitted
+// tuple's head: e_k(w) from the tuple's cursor over its exact receives (the
+// cursor only moves forward because wildcards of a tuple are visited in
+// posting order), plus the claims c_k; redux.sync.min takes the earliest
+// arrival and the winning tuple logs the claim.
+template <class CandF>
+__device__ __forceinline__ void resolve_wildcard(const FifoWs& ws, uint32_t w, uint64_t r, uint64_t msk, uint32_t nc,
+                                                 CandF cand, int lane) {
+  uint32_t best = 0xFFFFFFFFu, bestk = 0;
+  for (uint32_t c0 = lane; c0 < nc; c0 += 32) {
+    const uint32_t k = cand(c0);
+    if (((ws.keyhdr[k] ^ r) & msk) == 0) {
+      uint32_t cur = ws.key_cur[k];
+      const uint32_t rs = ws.key_rstart[k], rc = ws.key_rcnt[k];
+      while (cur < rc && ws.rby_key[rs + cur] < w) cur++;
+      ws.key_cur[k] = (uint16_t)cur;
+      const uint32_t hd = cur + ws.key_c[k];
+      if (hd < ws.key_cnt[k]) {
+        const uint32_t j = ws.by_key[ws.key_start[k] + hd];
+        if (j < best) {
+          best = j;
+          bestk = k;
+        }
+      }
+    }
+  }
+  const uint32_t win = __reduce_min_sync(kFull, best);
+  if (win != 0xFFFFFFFFu && best == win) {
+    const uint32_t c = ws.key_c[bestk];
+    ws.wlog[ws.key_start[bestk] + c] = (uint16_t)w;
+    ws.key_c[bestk] = (uint16_t)(c + 1);
+  }
+  if (lane == 0) ws.recv_res[w] = win == 0xFFFFFFFFu ? kNone : (uint16_t)win;
+  __syncwarp();
 }
 
 template <int NT>
+__device__ __forceinline__ void stage_side(const Side& S, int e, int64_t n, int64_t res, int64_t pb, uint64_t* dst,
+                                           int tid) {
+  const uint64_t* q = S.q_hdr + (int64_t)e * S.cap;
+  if (((((uintptr_t)q) | ((uintptr_t)dst)) & 15) == 0) {
+    for (int64_t k = tid; k < (res >> 1); k += NT) reinterpret_cast<uint4*>(dst)[k] = reinterpret_cast<const uint4*>(q)[k];
+    if ((res & 1) && tid == 0) dst[res - 1] = q[res - 1];
+  } else {
+    for (int64_t k = tid; k < res; k += NT) dst[k] = q[k];
+  }
+  const int64_t np = n - res;
+  if (np <= 0) return;
+  const uint64_t* p = S.p_hdr + pb;
+  uint64_t* d = dst + res;
+  if (((((uintptr_t)p) | ((uintptr_t)d)) & 15) == 0) {
+    for (int64_t k = tid; k < (np >> 1); k += NT) reinterpret_cast<uint4*>(d)[k] = reinterpret_cast<const uint4*>(p)[k];
+    if ((np & 1) && tid == 0) d[np - 1] = p[np - 1];
+  } else {
+    for (int64_t k = tid; k < np; k += NT) d[k] = p[k];
+  }
+}
+
+// Ordered placement by one warp: element x (0..n) with tuple id key(x) (>=
+// kWild = skip) gets slot start[k] + running[k]; put(x, k, rank, slot).
+template <class KeyF, class PutF>
+__device__ __forceinline__ void place_in_order(int64_t n, KeyF key, const uint16_t* start, uint16_t* running, PutF put,
+                                               int lane, uint32_t lt) {
+  for (int64_t b = 0; b < n; b += 32) {
+    const int64_t x = b + lane;
+    const uint32_t k = x < n ? key(x) : 0xFFFFFFFFu;
+    const bool ok = k < kWild;
+    const uint32_t peers = __match_any_sync(kFull, ok ? k : 0xFFFFFFFFu);
+    uint32_t run = 0;
+    if (ok) run = running[k];
+    __syncwarp();
+    if (ok) {
+      const uint32_t r = run + __popc(peers & lt);
+      put(x, k, r, (uint32_t)start[k] + r);
+      if ((peers >> lane) == 1u) running[k] = (uint16_t)(run + __popc(peers));
+    }
+    __syncwarp();
+  }
+}
+
+template <int NT, bool SMEM>
 __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_t* gws) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   __shared__ uint32_t scan_sm[NT / 32 + 1];
-  __shared__ uint32_t sh_K;
-  uint8_t* base = L.in_smem ? smem_raw : gws + (size_t)blockIdx.x * L.total;
-  FifoWs ws = carve(base, L);
+  __shared__ uint32_t sh_K, sh_W, sh_matched, sh_types, sh_G;
+  // compile-time choice, so that shared-memory accesses compile to LDS/STS/ATOMS
+  uint8_t* base = SMEM ? smem_raw : gws + (size_t)blockIdx.x * L.total;
+  const FifoWs ws = carve(base, L);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t lt = lanemask_lt();
   const uint32_t H = L.H, hmask = L.H - 1;
@@ -109,56 +239,46 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       continue;  // uniform across the CTA
     }
 
-    // ---- 1. stage messages, clear the table -------------------------------
-    {
-      const uint64_t* q = a.M.q_hdr + (int64_t)e * a.M.cap;
-      for (int64_t k = tid; k < mres; k += NT) ws.msgs[k] = q[k];
-      const int64_t np = nm - mres;
-      const uint64_t* p = a.M.p_hdr ? a.M.p_hdr + mpb : nullptr;
-      uint64_t* d = ws.msgs + mres;
-      if (np > 0 && ((((uintptr_t)p) | ((uintptr_t)d)) & 15) == 0) {
-        for (int64_t k = tid; k < (np >> 1); k += NT)
-          reinterpret_cast<uint4*>(d)[k] = reinterpret_cast<const uint4*>(p)[k];
-        if ((np & 1) && tid == 0) d[np - 1] = p[np - 1];
-      } else {
-        for (int64_t k = tid; k < np; k += NT) d[k] = p[k];
-      }
-      for (uint32_t s = tid; s < H / 2; s += NT) reinterpret_cast<uint32_t*>(ws.table)[s] = 0xFFFFFFFFu;
-      for (int64_t k = tid; k < (nm + 31) / 32; k += NT) ws.matched[k] = 0u;
-    }
+    // P1 -------------------------------------------------------------------
+    stage_side<NT>(a.M, e, nm, mres, mpb, ws.msgs, tid);
+    stage_side<NT>(a.R, e, nr, rres, rpb, ws.recvs, tid);
+    for (uint32_t s = tid; s < H / 2; s += NT) reinterpret_cast<uint32_t*>(ws.table)[s] = 0xFFFFFFFFu;
+    for (int64_t k = tid; k < (nm + 31) / 32; k += NT) ws.matched[k] = 0u;
+    if (tid == 0) sh_matched = 0;
     __syncthreads();
-    // insert every message's tuple (linear probing, lock-free)
+    // P2 -------------------------------------------------------------------
     for (int64_t j = tid; j < nm; j += NT) {
       const uint64_t h = ws.msgs[j];
       uint32_t s = header_hash(h) & hmask;
       while (true) {
         uint16_t o = ws.table[s];
-        if (o == kSlotEmpty) {
-          o = cas16(&ws.table[s], kSlotEmpty, (uint16_t)j);
-          if (o == kSlotEmpty) break;
+        if (o == kEmpty16) {
+          o = cas16(&ws.table[s], kEmpty16, (uint16_t)j);
+          if (o == kEmpty16) break;
         }
         if (ws.msgs[o] == h) break;
         s = (s + 1) & hmask;
       }
-      ws.msg_key[j] = s;
+      ws.msg_key[j] = (uint16_t)s;
     }
     __syncthreads();
-    // dense tuple ids in slot order
+    // P3 -------------------------------------------------------------------
     {
       const uint32_t per = (H + NT - 1) / NT;
-      const uint32_t s0 = tid * per, s1 = min(H, s0 + per);
+      const uint32_t s0 = min(H, tid * per), s1 = min(H, s0 + per);
       uint32_t c = 0;
-      for (uint32_t s = s0; s < s1; s++) c += ws.table[s] != kSlotEmpty;
+      for (uint32_t s = s0; s < s1; s++) c += ws.table[s] != kEmpty16;
       uint32_t tot;
-      uint32_t id = block_scan_u32<NT>(c, scan_sm, &tot);
+      uint32_t id = block_excl_scan<uint32_t>(c, scan_sm, &tot);
       for (uint32_t s = s0; s < s1; s++) {
         const uint16_t o = ws.table[s];
-        if (o != kSlotEmpty) {
+        if (o != kEmpty16) {
           ws.slot_id[s] = (uint16_t)id;
-          ws.key_owner[id] = o;
+          ws.keyhdr[id] = ws.msgs[o];
           ws.key_cnt[id] = 0;
-          ws.key_e[id] = 0;
+          ws.key_rcnt[id] = 0;
           ws.key_c[id] = 0;
+          ws.key_cur[id] = 0;
           id++;
         }
       }
@@ -166,186 +286,268 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     }
     __syncthreads();
     const uint32_t K = sh_K;
+    // P4 -------------------------------------------------------------------
     for (int64_t j = tid; j < nm; j += NT) {
-      const uint32_t id = ws.slot_id[ws.msg_key[j]];
+      const uint16_t id = ws.slot_id[ws.msg_key[j]];
       ws.msg_key[j] = id;
-      atomicAdd(&ws.key_cnt[id], 1u);
+      inc16(&ws.key_cnt[id]);
+    }
+    for (int64_t i = tid; i < nr; i += NT) {
+      const uint64_t h = ws.recvs[i];
+      uint16_t rk;
+      if (wildcard_mask(h) != ~0ull) {
+        rk = kWild;
+      } else {
+        rk = kNone;
+        uint32_t s = header_hash(h) & hmask;
+        while (true) {
+          const uint16_t o = ws.table[s];
+          if (o == kEmpty16) break;
+          if (ws.msgs[o] == h) {
+            rk = ws.slot_id[s];
+            break;
+          }
+          s = (s + 1) & hmask;
+        }
+        if (rk != kNone) inc16(&ws.key_rcnt[rk]);
+      }
+      ws.recv_key[i] = rk;
     }
     __syncthreads();
+    // P5 -------------------------------------------------------------------
     {
+      // tuple list starts for messages (low half) and exact receives (high)
       const uint32_t per = (K + NT - 1) / NT;
       const uint32_t k0 = min(K, tid * per), k1 = min(K, k0 + per);
       uint32_t c = 0;
-      for (uint32_t k = k0; k < k1; k++) c += ws.key_cnt[k];
+      for (uint32_t k = k0; k < k1; k++) c += (uint32_t)ws.key_cnt[k] | ((uint32_t)ws.key_rcnt[k] << 16);
       uint32_t tot;
-      uint32_t st = block_scan_u32<NT>(c, scan_sm, &tot);
+      uint32_t st = block_excl_scan<uint32_t>(c, scan_sm, &tot);
       for (uint32_t k = k0; k < k1; k++) {
-        ws.key_start[k] = st;
-        st += ws.key_cnt[k];
+        ws.key_start[k] = (uint16_t)st;
+        ws.key_rstart[k] = (uint16_t)(st >> 16);
+        st += (uint32_t)ws.key_cnt[k] | ((uint32_t)ws.key_rcnt[k] << 16);
       }
+      // ordered list of wildcard receives
+      const uint32_t rper = (uint32_t)((nr + NT - 1) / NT);
+      const uint32_t i0 = (uint32_t)min((int64_t)tid * rper, nr), i1 = (uint32_t)min((int64_t)i0 + rper, nr);
+      uint32_t wc = 0;
+      for (uint32_t i = i0; i < i1; i++) wc += ws.recv_key[i] == kWild;
+      uint32_t wt;
+      uint32_t wp = block_excl_scan<uint32_t>(wc, scan_sm, &wt);
+      for (uint32_t i = i0; i < i1 && wc; i++)
+        if (ws.recv_key[i] == kWild) ws.wl[wp++] = (uint16_t)i;
+      if (tid == 0) sh_W = wt;
     }
     __syncthreads();
+    const uint32_t W = sh_W;
+    // P6 -------------------------------------------------------------------
     if (warp == 0) {
-      // place messages into their tuple lists in arrival order (key_e is the
-      // running count here and is cleared again below)
-      for (int64_t b = 0; b < nm; b += 32) {
-        const int64_t j = b + lane;
-        const uint32_t id = j < nm ? ws.msg_key[j] : 0xFFFFFFFFu;
-        const uint32_t peers = __match_any_sync(kFull, id);
-        if (j < nm) {
-          const uint32_t run = ws.key_e[id];
-          ws.by_key[ws.key_start[id] + run + __popc(peers & lt)] = (uint16_t)j;
-          __syncwarp(peers);
-          if ((peers >> lane) == 1u) ws.key_e[id] = run + __popc(peers);
-        }
-        __syncwarp();
+      place_in_order(
+          nm, [&](int64_t j) { return (uint32_t)ws.msg_key[j]; }, ws.key_start, ws.key_cur,
+          [&](int64_t j, uint32_t, uint32_t, uint32_t slot) { ws.by_key[slot] = (uint16_t)j; }, lane, lt);
+    } else if (warp == 1) {
+      place_in_order(
+          nr, [&](int64_t i) { return (uint32_t)ws.recv_key[i]; }, ws.key_rstart, ws.key_c,
+          [&](int64_t i, uint32_t, uint32_t r, uint32_t slot) {
+            ws.rby_key[slot] = (uint16_t)i;
+            ws.recv_e[i] = (uint16_t)r;
+          },
+          lane, lt);
+    }
+    __syncthreads();
+    for (uint32_t k = tid; k < K; k += NT) {
+      ws.key_c[k] = 0;
+      ws.key_cur[k] = 0;
+    }
+    __syncthreads();
+    // P7: wildcards -------------------------------------------------------
+    if (W > 0) {
+      // Wildcards of one type (all ANY_SOURCE, all ANY_TAG, or all both) touch
+      // disjoint tuple groups {k : k & mask == r & mask}; groups are then
+      // independent and are processed by different warps, each group's
+      // wildcards in posting order.  Mixed types fall back to one warp.
+      if (tid == 0) sh_types = 0;
+      __syncthreads();
+      for (uint32_t x = tid; x < W; x += NT) {
+        const uint64_t r = ws.recvs[ws.wl[x]];
+        const uint32_t code = ((uint32_t)r == MM_ANY_SOURCE ? 1u : 0u) |
+                              (((uint32_t)(r >> 32) & 0xFFFFu) == MM_ANY_TAG ? 2u : 0u);
+        atomicOr(&sh_types, 1u << code);
       }
-    } else {
-      // classify receives: exact tuple id, wildcard, or a tuple no message has
-      for (int64_t i = tid - 32; i < nr; i += NT - 32) {
-        const uint64_t h = a.R.hdr(e, i, rres, rpb);
-        uint32_t rk;
-        if (wildcard_mask(h) != ~0ull) {
-          rk = kRecvWild;
-        } else {
-          rk = kRecvNone;
-          uint32_t s = header_hash(h) & hmask;
+      __syncthreads();
+      const uint32_t types = sh_types;
+      if (__popc(types) == 1 && K > 32) {
+        const uint32_t code = __ffs(types) - 1;
+        const uint64_t gmsk = (code & 1 ? ~0xFFFFFFFFull : ~0ull) & (code & 2 ? ~(0xFFFFull << 32) : ~0ull);
+        for (uint32_t s2 = tid; s2 < H / 2; s2 += NT) reinterpret_cast<uint32_t*>(ws.table)[s2] = 0xFFFFFFFFu;
+        __syncthreads();
+        for (uint32_t k = tid; k < K; k += NT) {
+          const uint64_t gk = ws.keyhdr[k] & gmsk;
+          uint32_t sl = header_hash(gk) & hmask;
           while (true) {
-            const uint16_t o = ws.table[s];
-            if (o == kSlotEmpty) break;
-            if (ws.msgs[o] == h) {
-              rk = ws.slot_id[s];
+            uint16_t o = ws.table[sl];
+            if (o == kEmpty16) {
+              o = cas16(&ws.table[sl], kEmpty16, (uint16_t)k);
+              if (o == kEmpty16) break;
+            }
+            if ((ws.keyhdr[o] & gmsk) == gk) break;
+            sl = (sl + 1) & hmask;
+          }
+          ws.key_grp[k] = (uint16_t)sl;
+        }
+        __syncthreads();
+        {
+          const uint32_t per = (H + NT - 1) / NT;
+          const uint32_t s0 = min(H, tid * per), s1 = min(H, s0 + per);
+          uint32_t c = 0;
+          for (uint32_t q = s0; q < s1; q++) c += ws.table[q] != kEmpty16;
+          uint32_t tot;
+          uint32_t id = block_excl_scan<uint32_t>(c, scan_sm, &tot);
+          for (uint32_t q = s0; q < s1; q++)
+            if (ws.table[q] != kEmpty16) {
+              ws.slot_id[q] = (uint16_t)id;
+              ws.g_cnt[id] = 0;
+              ws.gw_cnt[id] = 0;
+              id++;
+            }
+          if (tid == 0) sh_G = tot;
+        }
+        __syncthreads();
+        const uint32_t G = sh_G;
+        for (uint32_t k = tid; k < K; k += NT) {
+          const uint16_t g = ws.slot_id[ws.key_grp[k]];
+          ws.key_grp[k] = g;
+          inc16(&ws.g_cnt[g]);
+        }
+        for (uint32_t x = tid; x < W; x += NT) {
+          const uint64_t rg = ws.recvs[ws.wl[x]] & gmsk;
+          uint32_t sl = header_hash(rg) & hmask;
+          uint16_t g = kNone;
+          while (true) {
+            const uint16_t o = ws.table[sl];
+            if (o == kEmpty16) break;
+            if ((ws.keyhdr[o] & gmsk) == rg) {
+              g = ws.slot_id[sl];
               break;
             }
-            s = (s + 1) & hmask;
+            sl = (sl + 1) & hmask;
+          }
+          ws.w_grp[x] = g;
+          ws.recv_res[ws.wl[x]] = kNone;  // no admissible tuple: stays unmatched
+          if (g != kNone) inc16(&ws.gw_cnt[g]);
+        }
+        __syncthreads();
+        {
+          const uint32_t per = (G + NT - 1) / NT;
+          const uint32_t g0 = min(G, tid * per), g1 = min(G, g0 + per);
+          uint32_t c = 0;
+          for (uint32_t g = g0; g < g1; g++) c += (uint32_t)ws.g_cnt[g] | ((uint32_t)ws.gw_cnt[g] << 16);
+          uint32_t tot;
+          uint32_t st = block_excl_scan<uint32_t>(c, scan_sm, &tot);
+          for (uint32_t g = g0; g < g1; g++) {
+            ws.g_start[g] = (uint16_t)st;
+            ws.gw_start[g] = (uint16_t)(st >> 16);
+            st += (uint32_t)ws.g_cnt[g] | ((uint32_t)ws.gw_cnt[g] << 16);
           }
         }
-        ws.recv_key[i] = rk;
+        __syncthreads();
+        for (uint32_t k = tid; k < K; k += NT) {
+          const uint32_t g = ws.key_grp[k];
+          ws.g_keys[ws.g_start[g] + fetch_inc16(&ws.key_cur[g])] = (uint16_t)k;  // order within a group is free
+        }
+        if (warp == NT / 32 - 1)
+          place_in_order(
+              (int64_t)W, [&](int64_t x) { return (uint32_t)ws.w_grp[x]; }, ws.gw_start, ws.key_c,
+              [&](int64_t x, uint32_t, uint32_t, uint32_t slot) { ws.gw_list[slot] = (uint16_t)x; }, lane, lt);
+        __syncthreads();
+        for (uint32_t k = tid; k < K; k += NT) {
+          ws.key_c[k] = 0;
+          ws.key_cur[k] = 0;
+        }
+        __syncthreads();
+        for (uint32_t g = warp; g < G; g += NT / 32) {
+          const uint32_t ws0 = ws.gw_start[g], wn = ws.gw_cnt[g];
+          const uint32_t ks0 = ws.g_start[g], kn = ws.g_cnt[g];
+          for (uint32_t t = 0; t < wn; t++) {
+            const uint32_t w = ws.wl[ws.gw_list[ws0 + t]];
+            const uint64_t r = ws.recvs[w];
+            resolve_wildcard(ws, w, r, wildcard_mask(r), kn, [&](uint32_t c0) { return (uint32_t)ws.g_keys[ks0 + c0]; },
+                             lane);
+          }
+        }
+      } else if (warp == 0) {
+        for (uint32_t x = 0; x < W; x++) {
+          const uint32_t w = ws.wl[x];
+          const uint64_t r = ws.recvs[w];
+          resolve_wildcard(ws, w, r, wildcard_mask(r), K, [](uint32_t c0) { return c0; }, lane);
+        }
       }
     }
     __syncthreads();
-    for (uint32_t k = tid; k < K; k += NT) ws.key_e[k] = 0;
-    __syncthreads();
-
-    // ---- 2. in-order sweep (one warp) --------------------------------------
-    if (warp == 0) {
+    // P8: resolve receives, write results, compact the posted-receive queue --
+    {
       uint64_t* qrh = a.q_rh_w + (int64_t)e * a.R.cap;
       int64_t* qrc = a.q_rc_w + (int64_t)e * a.R.cap;
-      int64_t wr = 0;
-      uint32_t nmatch = 0;
-      // software pipeline: the next chunk's headers/cookies are in flight
-      // while the current chunk resolves
-      uint64_t nrh = 0;
-      int64_t nrc = 0;
-      if (lane < nr) {
-        nrh = a.R.hdr(e, lane, rres, rpb);
-        nrc = a.R.cookie(e, lane, rres, rpb);
-      }
-      for (int64_t b0 = 0; b0 < nr; b0 += 32) {
-        const int64_t i = b0 + lane;
+      uint32_t wr = 0, nmatch = 0;
+      for (int64_t b0 = 0; b0 < nr; b0 += NT) {
+        const int64_t i = b0 + tid;
         const bool valid = i < nr;
-        const uint64_t rh = nrh;
-        const int64_t rc = nrc;
-        if (i + 32 < nr) {
-          nrh = a.R.hdr(e, i + 32, rres, rpb);
-          nrc = a.R.cookie(e, i + 32, rres, rpb);
-        }
-        const uint32_t rk = valid ? ws.recv_key[i] : kRecvNone;
-        int64_t res = -1;
-        uint32_t wmask = __ballot_sync(kFull, valid && rk == kRecvWild);
-        int seg = 0;
-        while (true) {
-          const int t = wmask ? __ffs(wmask) - 1 : 32;
-          // exact receives in lanes [seg, t)
-          const bool in = valid && lane >= seg && lane < t && rk < kRecvWild;
-          const uint32_t key = in ? rk : 0xFFFFFFFFu;
-          const uint32_t peers = __match_any_sync(kFull, key);
-          uint32_t e0 = 0;
-          if (in) {
-            e0 = ws.key_e[rk];
-            const uint32_t hd = e0 + __popc(peers & lt) + ws.key_c[rk];
-            if (hd < ws.key_cnt[rk]) {
-              const uint32_t j = ws.by_key[ws.key_start[rk] + hd];
-              res = j;
-              atomicOr(&ws.matched[j >> 5], 1u << (j & 31));
-            }
-          }
-          __syncwarp();
-          if (in && (peers >> lane) == 1u) ws.key_e[rk] = e0 + __popc(peers);
-          __syncwarp();
-          if (t == 32) break;
-          // wildcard receive at lane t: earliest head among admitted tuples
-          const uint64_t r = __shfl_sync(kFull, rh, t);
-          const uint64_t msk = wildcard_mask(r);
-          uint32_t best = 0xFFFFFFFFu, bestk = 0;
-          for (uint32_t k = lane; k < K; k += 32) {
-            if (((ws.msgs[ws.key_owner[k]] ^ r) & msk) == 0) {
-              const uint32_t hd = ws.key_e[k] + ws.key_c[k];
-              if (hd < ws.key_cnt[k]) {
-                const uint32_t j = ws.by_key[ws.key_start[k] + hd];
-                if (j < best) {
-                  best = j;
-                  bestk = k;
-                }
-              }
-            }
-          }
-          const uint32_t win = __reduce_min_sync(kFull, best);
-          if (win != 0xFFFFFFFFu) {
-            if (best == win) {
-              ws.key_c[bestk] += 1;
-              atomicOr(&ws.matched[win >> 5], 1u << (win & 31));
-            }
-            if (lane == t) res = win;
-          }
-          __syncwarp();
-          wmask &= ~(1u << t);
-          seg = t + 1;
-        }
+        uint32_t res = kNone;
+        int64_t rc = 0;
         if (valid) {
+          rc = a.R.cookie(e, i, rres, rpb);
+          const uint16_t rk = ws.recv_key[i];
+          if (rk == kWild) {
+            res = ws.recv_res[i];
+          } else if (rk != kNone) {
+            const uint32_t st = ws.key_start[rk], nc = ws.key_c[rk];
+            uint32_t c = 0;
+            while (c < nc && ws.wlog[st + c] < i) c++;  // claims before i (ascending)
+            const uint32_t hd = (uint32_t)ws.recv_e[i] + c;
+            if (hd < ws.key_cnt[rk]) res = ws.by_key[st + hd];
+          }
+          if (res != kNone) atomicOr(&ws.matched[res >> 5], 1u << (res & 31));
           a.out_rc[obase + i] = rc;
-          a.out_mc[obase + i] = res >= 0 ? a.M.cookie(e, res, mres, mpb) : (int64_t)MM_NO_MATCH;
+          a.out_mc[obase + i] = res != kNone ? a.M.cookie(e, res, mres, mpb) : (int64_t)MM_NO_MATCH;
         }
-        const uint32_t um = __ballot_sync(kFull, valid && res < 0);
-        nmatch += __popc(__ballot_sync(kFull, valid && res >= 0));
-        __syncwarp();
-        if (valid && res < 0) {
-          const int64_t pos = wr + __popc(um & lt);
-          qrh[pos] = rh;
+        const uint32_t um = (valid && res == kNone) ? 1u : 0u;
+        nmatch += (valid && res != kNone) ? 1u : 0u;
+        uint32_t tot;
+        const uint32_t pos = wr + block_excl_scan<uint32_t>(um, scan_sm, &tot);  // syncs: reads precede writes
+        if (um) {
+          qrh[pos] = ws.recvs[i];
           qrc[pos] = rc;
         }
-        wr += __popc(um);
+        wr += tot;
       }
-      if (lane == 0) {
-        a.rres_w[e] = (int32_t)wr;
-        if (nmatch) atomicAdd(a.n_matched, (unsigned long long)nmatch);
-      }
+      for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
+      if (lane == 0 && nmatch) atomicAdd(&sh_matched, nmatch);
+      if (tid == 0) a.rres_w[e] = (int32_t)wr;
     }
     __syncthreads();
-    // ---- 3. compact the unexpected-message queue (warp 1, or 0) -----------
-    if (warp == (NT > 32 ? 1 : 0)) {
+    // P9: compact the unexpected-message queue ------------------------------
+    {
       uint64_t* qmh = a.q_mh_w + (int64_t)e * a.M.cap;
       int64_t* qmc = a.q_mc_w + (int64_t)e * a.M.cap;
-      int64_t wm = 0;
-      for (int64_t b0 = 0; b0 < nm; b0 += 32) {
-        const int64_t j = b0 + lane;
+      uint32_t wm = 0;
+      for (int64_t b0 = 0; b0 < nm; b0 += NT) {
+        const int64_t j = b0 + tid;
         const bool keep = j < nm && !((ws.matched[j >> 5] >> (j & 31)) & 1u);
-        uint64_t h = 0;
         int64_t c = 0;
+        if (keep) c = a.M.cookie(e, j, mres, mpb);
+        uint32_t tot;
+        const uint32_t pos = wm + block_excl_scan<uint32_t>(keep ? 1u : 0u, scan_sm, &tot);
         if (keep) {
-          h = ws.msgs[j];
-          c = a.M.cookie(e, j, mres, mpb);
-        }
-        const uint32_t km = __ballot_sync(kFull, keep);
-        __syncwarp();
-        if (keep) {
-          const int64_t pos = wm + __popc(km & lt);
-          qmh[pos] = h;
+          qmh[pos] = ws.msgs[j];
           qmc[pos] = c;
         }
-        wm += __popc(km);
+        wm += tot;
       }
-      if (lane == 0) a.mres_w[e] = (int32_t)wm;
+      if (tid == 0) {
+        a.mres_w[e] = (int32_t)wm;
+        if (sh_matched) atomicAdd(a.n_matched, (unsigned long long)sh_matched);
+      }
     }
     __syncthreads();  // the workspace is reused by the next endpoint
   }
@@ -364,17 +566,33 @@ FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
     return o;
   };
   L.msgs = take(8 * mcap);
+  L.recvs = take(8 * rcap);
+  L.keyhdr = take(8 * mcap);
   L.table = take(2 * H);
   L.slot_id = take(2 * H);
-  L.key_owner = take(2 * mcap);
-  L.key_cnt = take(4 * mcap);
-  L.key_start = take(4 * mcap);
-  L.key_e = take(4 * mcap);
-  L.key_c = take(4 * mcap);
-  L.msg_key = take(4 * mcap);
+  L.key_cnt = take(2 * mcap);
+  L.key_start = take(2 * mcap);
+  L.key_rcnt = take(2 * mcap);
+  L.key_rstart = take(2 * mcap);
+  L.key_c = take(2 * mcap);
+  L.key_cur = take(2 * mcap);
+  L.msg_key = take(2 * mcap);
   L.by_key = take(2 * mcap);
-  L.recv_key = take(4 * rcap);
+  L.wlog = take(2 * mcap);
+  L.recv_key = take(2 * rcap);
+  L.recv_e = take(2 * rcap);
+  L.rby_key = take(2 * rcap);
+  L.recv_res = take(2 * rcap);
+  L.wl = take(2 * rcap);
   L.matched = take(4 * ((mcap + 31) / 32));
+  L.key_grp = take(2 * mcap);
+  L.g_cnt = take(2 * mcap);
+  L.g_start = take(2 * mcap);
+  L.g_keys = take(2 * mcap);
+  L.gw_cnt = take(2 * mcap);
+  L.gw_start = take(2 * mcap);
+  L.w_grp = take(2 * rcap);
+  L.gw_list = take(2 * rcap);
   L.total = off;
   L.in_smem = off <= kFifoSmemMax;
   return L;
@@ -391,13 +609,13 @@ cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws,
   const int grid = fifo_grid(L, a.n_ep);
   cudaError_t err;
   if (L.in_smem) {
-    err = cudaFuncSetAttribute(k_mpi_fifo<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
+    err = cudaFuncSetAttribute(k_mpi_fifo<256, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
     if (err != cudaSuccess) return err;
     count_launch();
-    k_mpi_fifo<128><<<grid, 128, (size_t)L.total, st>>>(a, L, nullptr);
+    k_mpi_fifo<256, true><<<grid, 256, (size_t)L.total, st>>>(a, L, nullptr);
   } else {
     count_launch();
-    k_mpi_fifo<512><<<grid, 512, 0, st>>>(a, L, gws);
+    k_mpi_fifo<512, false><<<grid, 512, 0, st>>>(a, L, gws);
   }
   return cudaGetLastError();
 }

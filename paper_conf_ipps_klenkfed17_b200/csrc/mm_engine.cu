@@ -240,7 +240,8 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
   if (semantics < MM_SEM_MPI || semantics > MM_SEM_NOWILD_UNORDERED) return MM_ERR_ARG;
   if (n_endpoints < 1 || recv_capacity < 1 || msg_capacity < 1) return MM_ERR_ARG;
   if (semantics != MM_SEM_MPI && n_endpoints != 1) return MM_ERR_ARG;
-  if (semantics == MM_SEM_MPI && msg_capacity > MM_MPI_MAX_MSGS) return MM_ERR_ARG;
+  if (semantics == MM_SEM_MPI && (msg_capacity > MM_MPI_MAX_MSGS || recv_capacity > MM_MPI_MAX_RECVS))
+    return MM_ERR_ARG;
   if (semantics != MM_SEM_MPI && recv_capacity + msg_capacity >= (int64_t)1 << 31) return MM_ERR_ARG;
   mm_engine* e = new (std::nothrow) mm_engine();
   if (!e) return MM_ERR_NOMEM;
