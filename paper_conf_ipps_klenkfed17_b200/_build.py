@@ -35,20 +35,24 @@ def stale():
     return any(os.path.getmtime(f) > t for f in _inputs())
 
 
-def build_library(force=False, verbose=False):
-    """Compile every csrc/*.cu into lib/libmm.so (sm_100a, -lineinfo)."""
-    if not force and not stale():
+def build_library(force=False, verbose=False, variant=""):
+    """Compile every csrc/*.cu into lib/libmm.so (sm_100a, -lineinfo).
+    variant="timing" builds lib/libmm_timing.so with -DMM_PHASE_TIMING
+    (per-phase clock64 accounting, a profiling aid only)."""
+    lib = LIB if not variant else os.path.join(LIBDIR, "libmm_%s.so" % variant)
+    if not force and not variant and not stale():
         return LIB
     os.makedirs(LIBDIR, exist_ok=True)
     nvcc = os.environ.get("NVCC", "nvcc")
-    tmp = LIB + ".tmp%d" % os.getpid()
-    cmd = [nvcc, *NVCC_FLAGS, "-Xptxas", "-v", "-o", tmp, *sources()]
+    tmp = lib + ".tmp%d" % os.getpid()
+    extra = ["-DMM_PHASE_TIMING"] if variant == "timing" else []
+    cmd = [nvcc, *NVCC_FLAGS, *extra, "-Xptxas", "-v", "-o", tmp, *sources()]
     res = subprocess.run(cmd, capture_output=True, text=True)
-    with open(os.path.join(LIBDIR, "ptxas.log"), "w") as f:
+    with open(os.path.join(LIBDIR, "ptxas%s.log" % ("_" + variant if variant else "")), "w") as f:
         f.write(" ".join(cmd) + "\n" + res.stdout + res.stderr)
     if res.returncode != 0:
         raise RuntimeError("nvcc failed:\n" + res.stderr[-4000:])
-    os.replace(tmp, LIB)
+    os.replace(tmp, lib)
     if verbose:
-        print("built", LIB)
-    return LIB
+        print("built", lib)
+    return lib

@@ -69,8 +69,8 @@ def load(build_if_missing=True):
     global _lib
     if _lib is not None:
         return _lib
-    path = _build.LIB
-    if build_if_missing and _build.stale():
+    path = os.environ.get("MM_LIB", _build.LIB)  # MM_LIB: profiling builds only
+    if build_if_missing and path == _build.LIB and _build.stale():
         _build.build_library()
     if not os.path.exists(path):
         raise RuntimeError("libmm.so not found at %s: the CUDA extension is required "

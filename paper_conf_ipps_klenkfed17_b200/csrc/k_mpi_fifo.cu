@@ -35,6 +35,24 @@
 
 namespace mm {
 
+// Optional per-phase cycle accounting (build with -DMM_PHASE_TIMING; read by
+// mm_debug_phase_cycles).  Thread 0 of each CTA adds clock64 deltas.
+#ifdef MM_PHASE_TIMING
+__device__ unsigned long long g_phase_cycles[16];
+#define MM_PHASE(n)                                                      \
+  do {                                                                  \
+    if (threadIdx.x == 0) {                                             \
+      const long long _t = clock64();                                   \
+      atomicAdd(&g_phase_cycles[n], (unsigned long long)(_t - t_phase)); \
+      t_phase = _t;                                                     \
+    }                                                                   \
+  } while (0)
+#else
+#define MM_PHASE(n) \
+  do {              \
+  } while (0)
+#endif
+
 constexpr uint16_t kWild = 0xFFFEu;
 constexpr uint16_t kNone = 0xFFFFu;
 constexpr uint16_t kEmpty16 = 0xFFFFu;
@@ -69,6 +87,8 @@ struct FifoWs {
   uint16_t* gw_start;   // [mcap] start of group g in gw_list
   uint16_t* w_grp;      // [rcap] wildcard (index into wl) -> group | kNone
   uint16_t* gw_list;    // [rcap] wildcards grouped by group, posting order
+  uint16_t* pcnt;       // [8][mcap] per-quarter tuple counts (aliases the group arrays)
+  int64_t mcap;         // row stride of pcnt
 };
 
 __device__ __forceinline__ FifoWs carve(uint8_t* base, const FifoLayout& L) {
@@ -101,6 +121,8 @@ __device__ __forceinline__ FifoWs carve(uint8_t* base, const FifoLayout& L) {
   w.gw_start = reinterpret_cast<uint16_t*>(base + L.gw_start);
   w.w_grp = reinterpret_cast<uint16_t*>(base + L.w_grp);
   w.gw_list = reinterpret_cast<uint16_t*>(base + L.gw_list);
+  w.pcnt = reinterpret_cast<uint16_t*>(base + L.pcnt);
+  w.mcap = L.mcap;
   return w;
 }
 
@@ -195,16 +217,31 @@ __device__ __forceinline__ void stage_side(const Side& S, int e, int64_t n, int6
   }
 }
 
+// Lanes holding the same value as this lane, from one ballot per value bit
+// (nbits covers every value in play).  Replaces match.any, whose cost grows
+// with the number of distinct values in the warp.
+__device__ __forceinline__ uint32_t peers_of(uint32_t v, int nbits) {
+  uint32_t m = kFull;
+  for (int b = 0; b < nbits; b++) {
+    const bool bit = (v >> b) & 1u;
+    const uint32_t bb = __ballot_sync(kFull, bit);
+    m &= bit ? bb : ~bb;
+  }
+  return m;
+}
+
 // Ordered placement by one warp: element x (0..n) with tuple id key(x) (>=
 // kWild = skip) gets slot start[k] + running[k]; put(x, k, rank, slot).
+// nkeys bounds the tuple ids (ids < nkeys).
 template <class KeyF, class PutF>
 __device__ __forceinline__ void place_in_order(int64_t n, KeyF key, const uint16_t* start, uint16_t* running, PutF put,
-                                               int lane, uint32_t lt) {
+                                               int lane, uint32_t lt, uint32_t nkeys) {
+  const int nbits = 32 - __clz(nkeys | 1u);  // ids 0..nkeys (nkeys = "skip")
   for (int64_t b = 0; b < n; b += 32) {
     const int64_t x = b + lane;
     const uint32_t k = x < n ? key(x) : 0xFFFFFFFFu;
     const bool ok = k < kWild;
-    const uint32_t peers = __match_any_sync(kFull, ok ? k : 0xFFFFFFFFu);
+    const uint32_t peers = peers_of(ok ? k : nkeys, nbits);
     uint32_t run = 0;
     if (ok) run = running[k];
     __syncwarp();
@@ -229,6 +266,9 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
   const uint32_t lt = lanemask_lt();
   const uint32_t H = L.H, hmask = L.H - 1;
 
+#ifdef MM_PHASE_TIMING
+  long long t_phase = clock64();
+#endif
   for (int e = blockIdx.x; e < a.n_ep; e += gridDim.x) {
     const int64_t rres = a.R.q_len[e], mres = a.M.q_len[e];
     const int64_t rpb = a.R.pend_begin(e), mpb = a.M.pend_begin(e);
@@ -238,6 +278,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       if (tid == 0) atomicOr(a.err, kErrCapacity);
       continue;  // uniform across the CTA
     }
+    MM_PHASE(0);
 
     // P1 -------------------------------------------------------------------
     stage_side<NT>(a.M, e, nm, mres, mpb, ws.msgs, tid);
@@ -246,6 +287,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     for (int64_t k = tid; k < (nm + 31) / 32; k += NT) ws.matched[k] = 0u;
     if (tid == 0) sh_matched = 0;
     __syncthreads();
+    MM_PHASE(1);
     // P2 -------------------------------------------------------------------
     for (int64_t j = tid; j < nm; j += NT) {
       const uint64_t h = ws.msgs[j];
@@ -262,6 +304,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       ws.msg_key[j] = (uint16_t)s;
     }
     __syncthreads();
+    MM_PHASE(2);
     // P3 -------------------------------------------------------------------
     {
       const uint32_t per = (H + NT - 1) / NT;
@@ -275,8 +318,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         if (o != kEmpty16) {
           ws.slot_id[s] = (uint16_t)id;
           ws.keyhdr[id] = ws.msgs[o];
-          ws.key_cnt[id] = 0;
-          ws.key_rcnt[id] = 0;
+#pragma unroll
+          for (int q = 0; q < 8; q++) ws.pcnt[q * ws.mcap + id] = 0;
           ws.key_c[id] = 0;
           ws.key_cur[id] = 0;
           id++;
@@ -286,11 +329,12 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     }
     __syncthreads();
     const uint32_t K = sh_K;
+    MM_PHASE(3);
     // P4 -------------------------------------------------------------------
     for (int64_t j = tid; j < nm; j += NT) {
       const uint16_t id = ws.slot_id[ws.msg_key[j]];
       ws.msg_key[j] = id;
-      inc16(&ws.key_cnt[id]);
+      inc16(&ws.pcnt[(int64_t)((j * 4) / nm) * ws.mcap + id]);
     }
     for (int64_t i = tid; i < nr; i += NT) {
       const uint64_t h = ws.recvs[i];
@@ -309,18 +353,33 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           }
           s = (s + 1) & hmask;
         }
-        if (rk != kNone) inc16(&ws.key_rcnt[rk]);
+        if (rk != kNone) inc16(&ws.pcnt[(4 + (int64_t)((i * 4) / nr)) * ws.mcap + rk]);
       }
       ws.recv_key[i] = rk;
     }
     __syncthreads();
+    MM_PHASE(4);
     // P5 -------------------------------------------------------------------
     {
       // tuple list starts for messages (low half) and exact receives (high)
       const uint32_t per = (K + NT - 1) / NT;
       const uint32_t k0 = min(K, tid * per), k1 = min(K, k0 + per);
       uint32_t c = 0;
-      for (uint32_t k = k0; k < k1; k++) c += (uint32_t)ws.key_cnt[k] | ((uint32_t)ws.key_rcnt[k] << 16);
+      for (uint32_t k = k0; k < k1; k++) {
+        // exclusive prefix over the quarters: the base rank of each quarter
+        uint32_t rm = 0, rr = 0;
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+          const uint32_t a = ws.pcnt[q * ws.mcap + k], b = ws.pcnt[(4 + q) * ws.mcap + k];
+          ws.pcnt[q * ws.mcap + k] = (uint16_t)rm;
+          ws.pcnt[(4 + q) * ws.mcap + k] = (uint16_t)rr;
+          rm += a;
+          rr += b;
+        }
+        ws.key_cnt[k] = (uint16_t)rm;
+        ws.key_rcnt[k] = (uint16_t)rr;
+        c += rm | (rr << 16);
+      }
       uint32_t tot;
       uint32_t st = block_excl_scan<uint32_t>(c, scan_sm, &tot);
       for (uint32_t k = k0; k < k1; k++) {
@@ -341,26 +400,32 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     }
     __syncthreads();
     const uint32_t W = sh_W;
+    MM_PHASE(5);
     // P6 -------------------------------------------------------------------
-    if (warp == 0) {
-      place_in_order(
-          nm, [&](int64_t j) { return (uint32_t)ws.msg_key[j]; }, ws.key_start, ws.key_cur,
-          [&](int64_t j, uint32_t, uint32_t, uint32_t slot) { ws.by_key[slot] = (uint16_t)j; }, lane, lt);
-    } else if (warp == 1) {
-      place_in_order(
-          nr, [&](int64_t i) { return (uint32_t)ws.recv_key[i]; }, ws.key_rstart, ws.key_c,
-          [&](int64_t i, uint32_t, uint32_t r, uint32_t slot) {
-            ws.rby_key[slot] = (uint16_t)i;
-            ws.recv_e[i] = (uint16_t)r;
-          },
-          lane, lt);
+    // warps 0-3 place the four quarters of the messages, warps 4-7 the four
+    // quarters of the receives; each quarter starts from its base ranks
+    if (warp < 8) {
+      const bool msg_side = warp < 4;
+      const int q = warp & 3;
+      const int64_t n = msg_side ? nm : nr;
+      const int64_t x0 = (n * q + 3) / 4, x1 = (n * (q + 1) + 3) / 4;  // == ceil: x*4/n == q
+      uint16_t* running = ws.pcnt + (int64_t)warp * ws.mcap;
+      if (msg_side) {
+        place_in_order(
+            x1 - x0, [&](int64_t x) { return (uint32_t)ws.msg_key[x0 + x]; }, ws.key_start, running,
+            [&](int64_t x, uint32_t, uint32_t, uint32_t slot) { ws.by_key[slot] = (uint16_t)(x0 + x); }, lane, lt, K);
+      } else {
+        place_in_order(
+            x1 - x0, [&](int64_t x) { return (uint32_t)ws.recv_key[x0 + x]; }, ws.key_rstart, running,
+            [&](int64_t x, uint32_t, uint32_t r, uint32_t slot) {
+              ws.rby_key[slot] = (uint16_t)(x0 + x);
+              ws.recv_e[x0 + x] = (uint16_t)r;
+            },
+            lane, lt, K);
+      }
     }
     __syncthreads();
-    for (uint32_t k = tid; k < K; k += NT) {
-      ws.key_c[k] = 0;
-      ws.key_cur[k] = 0;
-    }
-    __syncthreads();
+    MM_PHASE(6);
     // P7: wildcards -------------------------------------------------------
     if (W > 0) {
       // Wildcards of one type (all ANY_SOURCE, all ANY_TAG, or all both) touch
@@ -459,7 +524,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         if (warp == NT / 32 - 1)
           place_in_order(
               (int64_t)W, [&](int64_t x) { return (uint32_t)ws.w_grp[x]; }, ws.gw_start, ws.key_c,
-              [&](int64_t x, uint32_t, uint32_t, uint32_t slot) { ws.gw_list[slot] = (uint16_t)x; }, lane, lt);
+              [&](int64_t x, uint32_t, uint32_t, uint32_t slot) { ws.gw_list[slot] = (uint16_t)x; }, lane, lt, G);
         __syncthreads();
         for (uint32_t k = tid; k < K; k += NT) {
           ws.key_c[k] = 0;
@@ -469,11 +534,46 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         for (uint32_t g = warp; g < G; g += NT / 32) {
           const uint32_t ws0 = ws.gw_start[g], wn = ws.gw_cnt[g];
           const uint32_t ks0 = ws.g_start[g], kn = ws.g_cnt[g];
-          for (uint32_t t = 0; t < wn; t++) {
-            const uint32_t w = ws.wl[ws.gw_list[ws0 + t]];
-            const uint64_t r = ws.recvs[w];
-            resolve_wildcard(ws, w, r, wildcard_mask(r), kn, [&](uint32_t c0) { return (uint32_t)ws.g_keys[ks0 + c0]; },
-                             lane);
+          if (wn == 0) continue;
+          if (kn <= 32) {
+            // every wildcard of the group has the same pattern and admits every
+            // tuple of the group: lane l owns tuple g_keys[l] and keeps its
+            // cursor and claim count in registers, so one wildcard costs a
+            // cursor step, one head read and one redux.
+            const bool own = lane < kn;
+            uint32_t k = 0, cur = 0, c = 0, rs = 0, rc = 0, st = 0, cnt = 0;
+            if (own) {
+              k = ws.g_keys[ks0 + lane];
+              rs = ws.key_rstart[k];
+              rc = ws.key_rcnt[k];
+              st = ws.key_start[k];
+              cnt = ws.key_cnt[k];
+            }
+            uint32_t nxt = ws.wl[ws.gw_list[ws0]];
+            for (uint32_t t = 0; t < wn; t++) {
+              const uint32_t w = nxt;
+              if (t + 1 < wn) nxt = ws.wl[ws.gw_list[ws0 + t + 1]];
+              uint32_t cand = 0xFFFFFFFFu;
+              if (own) {
+                while (cur < rc && ws.rby_key[rs + cur] < w) cur++;
+                const uint32_t hd = cur + c;
+                if (hd < cnt) cand = ws.by_key[st + hd];
+              }
+              const uint32_t win = __reduce_min_sync(kFull, cand);
+              if (win != 0xFFFFFFFFu && cand == win) {
+                ws.wlog[st + c] = (uint16_t)w;
+                c++;
+              }
+              if (lane == 0) ws.recv_res[w] = win == 0xFFFFFFFFu ? kNone : (uint16_t)win;
+            }
+            if (own) ws.key_c[k] = (uint16_t)c;
+          } else {
+            for (uint32_t t = 0; t < wn; t++) {
+              const uint32_t w = ws.wl[ws.gw_list[ws0 + t]];
+              const uint64_t r = ws.recvs[w];
+              resolve_wildcard(ws, w, r, wildcard_mask(r), kn,
+                               [&](uint32_t c0) { return (uint32_t)ws.g_keys[ks0 + c0]; }, lane);
+            }
           }
         }
       } else if (warp == 0) {
@@ -485,6 +585,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       }
     }
     __syncthreads();
+    MM_PHASE(7);
     // P8: resolve receives, write results, compact the posted-receive queue --
     {
       uint64_t* qrh = a.q_rh_w + (int64_t)e * a.R.cap;
@@ -526,6 +627,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       if (tid == 0) a.rres_w[e] = (int32_t)wr;
     }
     __syncthreads();
+    MM_PHASE(8);
     // P9: compact the unexpected-message queue ------------------------------
     {
       uint64_t* qmh = a.q_mh_w + (int64_t)e * a.M.cap;
@@ -550,6 +652,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       }
     }
     __syncthreads();  // the workspace is reused by the next endpoint
+    MM_PHASE(9);
   }
 }
 
@@ -559,12 +662,14 @@ FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
   while (H < 2 * mcap) H <<= 1;
   if (H < 64) H = 64;
   L.H = (uint32_t)H;
+  L.mcap = mcap;
   int64_t off = 0;
   auto take = [&](int64_t bytes) {
     int64_t o = off;
     off += (bytes + 15) / 16 * 16;
     return o;
   };
+  auto r16 = [](int64_t b) { return (b + 15) / 16 * 16; };
   L.msgs = take(8 * mcap);
   L.recvs = take(8 * rcap);
   L.keyhdr = take(8 * mcap);
@@ -576,23 +681,35 @@ FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
   L.key_rstart = take(2 * mcap);
   L.key_c = take(2 * mcap);
   L.key_cur = take(2 * mcap);
-  L.msg_key = take(2 * mcap);
+  // msg_key (P2..P6), w_grp (P7 set-up) and wlog (P7..P8) have disjoint lifetimes
+  L.msg_key = take(2 * (mcap > rcap ? mcap : rcap));
+  L.w_grp = L.msg_key;
+  L.wlog = L.msg_key;
   L.by_key = take(2 * mcap);
-  L.wlog = take(2 * mcap);
   L.recv_key = take(2 * rcap);
   L.recv_e = take(2 * rcap);
   L.rby_key = take(2 * rcap);
   L.recv_res = take(2 * rcap);
   L.wl = take(2 * rcap);
   L.matched = take(4 * ((mcap + 31) / 32));
-  L.key_grp = take(2 * mcap);
-  L.g_cnt = take(2 * mcap);
-  L.g_start = take(2 * mcap);
-  L.g_keys = take(2 * mcap);
-  L.gw_cnt = take(2 * mcap);
-  L.gw_start = take(2 * mcap);
-  L.w_grp = take(2 * rcap);
-  L.gw_list = take(2 * rcap);
+  // the per-quarter counts (P3..P6) share a region with the wildcard group
+  // arrays (P7 set-up and processing)
+  const int64_t grp = 6 * r16(2 * mcap) + r16(2 * rcap);
+  const int64_t region = take(grp > 16 * mcap ? grp : 16 * mcap);
+  L.pcnt = region;
+  int64_t g = region;
+  auto sub = [&](int64_t bytes) {
+    int64_t o = g;
+    g += r16(bytes);
+    return o;
+  };
+  L.key_grp = sub(2 * mcap);
+  L.g_cnt = sub(2 * mcap);
+  L.g_start = sub(2 * mcap);
+  L.g_keys = sub(2 * mcap);
+  L.gw_cnt = sub(2 * mcap);
+  L.gw_start = sub(2 * mcap);
+  L.gw_list = sub(2 * rcap);
   L.total = off;
   L.in_smem = off <= kFifoSmemMax;
   return L;
@@ -603,6 +720,18 @@ int fifo_grid(const FifoLayout& L, int n_ep) {
   int g = 148 * 2;
   return n_ep < g ? n_ep : g;
 }
+
+#ifdef MM_PHASE_TIMING
+extern "C" int mm_debug_phase_cycles(unsigned long long* out, int reset) {
+  cudaDeviceSynchronize();
+  if (cudaMemcpyFromSymbol(out, g_phase_cycles, sizeof(unsigned long long) * 16) != cudaSuccess) return 2;
+  if (reset) {
+    unsigned long long z[16] = {0};
+    cudaMemcpyToSymbol(g_phase_cycles, z, sizeof(z));
+  }
+  return 0;
+}
+#endif
 
 cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws, cudaStream_t st) {
   if (a.n_ep <= 0) return cudaSuccess;

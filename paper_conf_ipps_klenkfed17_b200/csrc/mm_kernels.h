@@ -29,7 +29,7 @@ constexpr int64_t kFifoSmemMax = 100 * 1024;
 struct FifoLayout {
   int64_t msgs, recvs, keyhdr, table, slot_id, key_cnt, key_start, key_rcnt, key_rstart, key_c, key_cur, msg_key, by_key,
       wlog, recv_key, recv_e, rby_key, recv_res, wl, matched, key_grp, g_cnt, g_start, g_keys, gw_cnt, gw_start,
-      w_grp, gw_list;
+      w_grp, gw_list, pcnt, mcap;
   int64_t total;
   uint32_t H;
   bool in_smem;
