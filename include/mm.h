@@ -197,8 +197,15 @@ int mm_route(const uint64_t *a, const int64_t *b, int64_t n, int32_t world, int3
  *   Both produce identical results.  Returns MM_ERR_ARG for unknown options
  *   or values.
  */
-enum { MM_OPT_MPI_KERNEL = 1 };
+enum { MM_OPT_MPI_KERNEL = 1, MM_OPT_FLAT_KERNEL = 2 };
 enum { MM_MPI_KERNEL_AUTO = 0, MM_MPI_KERNEL_MATRIX = 1, MM_MPI_KERNEL_FIFO = 2 };
+/*   MM_OPT_FLAT_KERNEL: how the no-wildcard levels run --
+ *     MM_FLAT_KERNEL_BUCKETED (default): hash-bucketed, one CTA per bucket in
+ *       shared memory; a batch with a bucket too large for
+ *       the chip (heavily repeated tuples) falls back to the global kernels;
+ *     MM_FLAT_KERNEL_GLOBAL: always the global kernels (LSD radix sort-and-rank
+ *       for NOWILD_ORDERED, HBM hash table for NOWILD_UNORDERED). */
+enum { MM_FLAT_KERNEL_BUCKETED = 0, MM_FLAT_KERNEL_GLOBAL = 1 };
 int mm_set_option(mm_engine *e, int32_t option, int64_t value);
 
 /* mm_strerror -- static description of an MM_* code. */

@@ -32,6 +32,7 @@
 //  P9 unmatched messages compacted in arrival order.
 // Exact by construction: no ties (arrival indices are unique).
 #include "mm_kernels.h"
+#include "mm_smem.cuh"
 
 namespace mm {
 
@@ -53,9 +54,6 @@ __device__ unsigned long long g_phase_cycles[16];
   } while (0)
 #endif
 
-constexpr uint16_t kWild = 0xFFFEu;
-constexpr uint16_t kNone = 0xFFFFu;
-constexpr uint16_t kEmpty16 = 0xFFFFu;
 
 struct FifoWs {
   uint64_t* msgs;       // [mcap] staged message headers
@@ -126,38 +124,6 @@ __device__ __forceinline__ FifoWs carve(uint8_t* base, const FifoLayout& L) {
   return w;
 }
 
-// 16-bit CAS through the containing 32-bit word.
-// (pointer arithmetic, not integer casts, so shared-memory provenance survives
-// and the atomics compile to ATOMS)
-__device__ __forceinline__ uint32_t* word_of(uint16_t* p) {
-  return reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(p) - (reinterpret_cast<uintptr_t>(p) & 2));
-}
-__device__ __forceinline__ uint16_t cas16(uint16_t* p, uint16_t expect, uint16_t val) {
-  uint32_t* w = word_of(p);
-  const uint32_t sh = (reinterpret_cast<uintptr_t>(p) & 2) ? 16u : 0u;
-  uint32_t old = *w;
-  while (true) {
-    const uint16_t cur = (uint16_t)(old >> sh);
-    if (cur != expect) return cur;
-    const uint32_t nw = (old & ~(0xFFFFu << sh)) | ((uint32_t)val << sh);
-    const uint32_t got = atomicCAS(w, old, nw);
-    if (got == old) return expect;
-    old = got;
-  }
-}
-
-// 16-bit counter increment through the containing 32-bit word (no carry out:
-// counts stay below 65536).
-__device__ __forceinline__ void inc16(uint16_t* p) {
-  atomicAdd(word_of(p), (reinterpret_cast<uintptr_t>(p) & 2) ? 0x10000u : 1u);
-}
-// Same, returning the previous 16-bit value.
-__device__ __forceinline__ uint32_t fetch_inc16(uint16_t* p) {
-  const bool hi = (reinterpret_cast<uintptr_t>(p) & 2) != 0;
-  const uint32_t old = atomicAdd(word_of(p), hi ? 0x10000u : 1u);
-  return hi ? (old >> 16) : (old & 0xFFFFu);
-}
-
 // One wildcard receive w (header r, mask msk) against candidate tuples
 // cand(0..nc) -- all admitted tuples are among them.  Lanes read each admitted
 // tuple's head: e_k(w) from the tuple's cursor over its exact receives (the
@@ -217,41 +183,54 @@ __device__ __forceinline__ void stage_side(const Side& S, int e, int64_t n, int6
   }
 }
 
-// Lanes holding the same value as this lane, from one ballot per value bit
-// (nbits covers every value in play).  Replaces match.any, whose cost grows
-// with the number of distinct values in the warp.
-__device__ __forceinline__ uint32_t peers_of(uint32_t v, int nbits) {
-  uint32_t m = kFull;
-  for (int b = 0; b < nbits; b++) {
-    const bool bit = (v >> b) & 1u;
-    const uint32_t bb = __ballot_sync(kFull, bit);
-    m &= bit ? bb : ~bb;
+// A chain of wildcard receives over at most 32 candidate tuples, one tuple per
+// lane with its cursor, claim count and head kept in registers: a wildcard
+// costs a compare, one redux.sync.min and (for the winner) one head reload.
+// test_admit: wildcards may differ, so each lane tests admission with the
+// masked XOR; otherwise every wildcard admits every candidate (a group).
+template <class KeyF, class PosF>
+__device__ __forceinline__ void register_chain(const FifoWs& ws, uint32_t kn, KeyF keyof, uint32_t wn, PosF posof,
+                                               bool test_admit, int lane) {
+  const bool own = lane < kn;
+  uint32_t k = 0, cur = 0, c = 0, rs = 0, rc = 0, st = 0, cnt = 0;
+  uint32_t nextpos = 0xFFFFFFFFu;  // posting position of the next exact receive of k
+  uint32_t head = 0xFFFFFFFFu;     // arrival index of k's first unclaimed message
+  uint64_t kh = 0;
+  if (own) {
+    k = keyof(lane);
+    rs = ws.key_rstart[k];
+    rc = ws.key_rcnt[k];
+    st = ws.key_start[k];
+    cnt = ws.key_cnt[k];
+    kh = ws.keyhdr[k];
+    if (rc > 0) nextpos = ws.rby_key[rs];
+    if (cnt > 0) head = ws.by_key[st];
   }
-  return m;
-}
-
-// Ordered placement by one warp: element x (0..n) with tuple id key(x) (>=
-// kWild = skip) gets slot start[k] + running[k]; put(x, k, rank, slot).
-// nkeys bounds the tuple ids (ids < nkeys).
-template <class KeyF, class PutF>
-__device__ __forceinline__ void place_in_order(int64_t n, KeyF key, const uint16_t* start, uint16_t* running, PutF put,
-                                               int lane, uint32_t lt, uint32_t nkeys) {
-  const int nbits = 32 - __clz(nkeys | 1u);  // ids 0..nkeys (nkeys = "skip")
-  for (int64_t b = 0; b < n; b += 32) {
-    const int64_t x = b + lane;
-    const uint32_t k = x < n ? key(x) : 0xFFFFFFFFu;
-    const bool ok = k < kWild;
-    const uint32_t peers = peers_of(ok ? k : nkeys, nbits);
-    uint32_t run = 0;
-    if (ok) run = running[k];
-    __syncwarp();
-    if (ok) {
-      const uint32_t r = run + __popc(peers & lt);
-      put(x, k, r, (uint32_t)start[k] + r);
-      if ((peers >> lane) == 1u) running[k] = (uint16_t)(run + __popc(peers));
+  uint32_t nxt = wn ? posof(0) : 0;
+  for (uint32_t t = 0; t < wn; t++) {
+    const uint32_t w = nxt;
+    if (t + 1 < wn) nxt = posof(t + 1);
+    if (nextpos < w) {  // exact receives of k posted before w consumed k's head(s)
+      do {
+        cur++;
+        nextpos = cur < rc ? ws.rby_key[rs + cur] : 0xFFFFFFFFu;
+      } while (nextpos < w);
+      head = cur + c < cnt ? ws.by_key[st + cur + c] : 0xFFFFFFFFu;
     }
-    __syncwarp();
+    uint32_t cand = head;
+    if (test_admit) {
+      const uint64_t r = ws.recvs[w];
+      if (((kh ^ r) & wildcard_mask(r)) != 0) cand = 0xFFFFFFFFu;
+    }
+    const uint32_t win = __reduce_min_sync(kFull, cand);
+    if (win != 0xFFFFFFFFu && cand == win) {
+      ws.wlog[st + c] = (uint16_t)w;
+      c++;
+      head = cur + c < cnt ? ws.by_key[st + cur + c] : 0xFFFFFFFFu;
+    }
+    if (lane == 0) ws.recv_res[w] = win == 0xFFFFFFFFu ? kNone : (uint16_t)win;
   }
+  if (own) ws.key_c[k] = (uint16_t)c;
 }
 
 template <int NT, bool SMEM>
@@ -442,7 +421,11 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       }
       __syncthreads();
       const uint32_t types = sh_types;
-      if (__popc(types) == 1 && K > 32) {
+      if (K <= 32) {
+        if (warp == 0)
+          register_chain(ws, K, [](uint32_t l) { return l; }, W, [&](uint32_t t) { return (uint32_t)ws.wl[t]; }, true,
+                         lane);
+      } else if (__popc(types) == 1) {
         const uint32_t code = __ffs(types) - 1;
         const uint64_t gmsk = (code & 1 ? ~0xFFFFFFFFull : ~0ull) & (code & 2 ? ~(0xFFFFull << 32) : ~0ull);
         for (uint32_t s2 = tid; s2 < H / 2; s2 += NT) reinterpret_cast<uint32_t*>(ws.table)[s2] = 0xFFFFFFFFu;
@@ -531,6 +514,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           ws.key_cur[k] = 0;
         }
         __syncthreads();
+        MM_PHASE(10);
         for (uint32_t g = warp; g < G; g += NT / 32) {
           const uint32_t ws0 = ws.gw_start[g], wn = ws.gw_cnt[g];
           const uint32_t ks0 = ws.g_start[g], kn = ws.g_cnt[g];
@@ -540,33 +524,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             // tuple of the group: lane l owns tuple g_keys[l] and keeps its
             // cursor and claim count in registers, so one wildcard costs a
             // cursor step, one head read and one redux.
-            const bool own = lane < kn;
-            uint32_t k = 0, cur = 0, c = 0, rs = 0, rc = 0, st = 0, cnt = 0;
-            if (own) {
-              k = ws.g_keys[ks0 + lane];
-              rs = ws.key_rstart[k];
-              rc = ws.key_rcnt[k];
-              st = ws.key_start[k];
-              cnt = ws.key_cnt[k];
-            }
-            uint32_t nxt = ws.wl[ws.gw_list[ws0]];
-            for (uint32_t t = 0; t < wn; t++) {
-              const uint32_t w = nxt;
-              if (t + 1 < wn) nxt = ws.wl[ws.gw_list[ws0 + t + 1]];
-              uint32_t cand = 0xFFFFFFFFu;
-              if (own) {
-                while (cur < rc && ws.rby_key[rs + cur] < w) cur++;
-                const uint32_t hd = cur + c;
-                if (hd < cnt) cand = ws.by_key[st + hd];
-              }
-              const uint32_t win = __reduce_min_sync(kFull, cand);
-              if (win != 0xFFFFFFFFu && cand == win) {
-                ws.wlog[st + c] = (uint16_t)w;
-                c++;
-              }
-              if (lane == 0) ws.recv_res[w] = win == 0xFFFFFFFFu ? kNone : (uint16_t)win;
-            }
-            if (own) ws.key_c[k] = (uint16_t)c;
+            register_chain(ws, kn, [&](uint32_t l) { return (uint32_t)ws.g_keys[ks0 + l]; }, wn,
+                           [&](uint32_t t) { return (uint32_t)ws.wl[ws.gw_list[ws0 + t]]; }, false, lane);
           } else {
             for (uint32_t t = 0; t < wn; t++) {
               const uint32_t w = ws.wl[ws.gw_list[ws0 + t]];

@@ -147,6 +147,9 @@ struct mm_engine {
   DBuf skey[2], sval[2], rid, run_start, run_rc, part;
   DBuf owner, rcnt, mcnt, tkey, tval;
   int64_t T = 0;
+  DBuf bh[4], bi[4], bpart, broff, bmoff, bover;
+  int flat_kernel = MM_FLAT_KERNEL_BUCKETED;
+  long long bucket_fallbacks = 0;
   Timer timer;
   long long launches = 0;
 };
@@ -227,7 +230,9 @@ int mm_destroy(mm_engine* e) {
   DBuf* bufs[] = {&e->out_off, &e->counts_dev, &e->nmatched, &e->err, &e->info, &e->out_rc_stage,
                   &e->out_mc_stage, &e->rflag, &e->mflag, &e->scan, &e->skey[0], &e->skey[1],
                   &e->sval[0], &e->sval[1], &e->rid, &e->run_start, &e->run_rc, &e->part,
-                  &e->owner, &e->rcnt, &e->mcnt, &e->tkey, &e->tval, &e->fifo_ws};
+                  &e->owner, &e->rcnt, &e->mcnt, &e->tkey, &e->tval, &e->fifo_ws,
+                  &e->bh[0], &e->bh[1], &e->bh[2], &e->bh[3], &e->bi[0], &e->bi[1], &e->bi[2], &e->bi[3],
+                  &e->bpart, &e->broff, &e->bmoff, &e->bover};
   for (DBuf* b : bufs) release(*b);
   delete e;
   return MM_OK;
@@ -275,6 +280,13 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
     const int64_t n = e->rcap + e->mcap;
     ok = ensure(e->rflag, e->rcap) == cudaSuccess && ensure(e->mflag, e->mcap) == cudaSuccess &&
          ensure(e->scan, (size_t)scan_scratch_elems(n) * 8) == cudaSuccess;
+    for (int b = 0; ok && b < 4; b++) {
+      const int64_t c = b < 2 ? e->rcap : e->mcap;
+      ok = ensure(e->bh[b], c * 8) == cudaSuccess && ensure(e->bi[b], c * 4) == cudaSuccess;
+    }
+    ok = ok && ensure(e->bpart, (size_t)partition_scratch_elems(e->rcap > e->mcap ? e->rcap : e->mcap) * 4) == cudaSuccess &&
+         ensure(e->broff, (size_t)bucket_scratch_elems(n) * 4) == cudaSuccess &&
+         ensure(e->bmoff, (size_t)bucket_scratch_elems(n) * 4) == cudaSuccess && ensure(e->bover, 4) == cudaSuccess;
     if (ok && semantics == MM_SEM_NOWILD_ORDERED) {
       ok = ensure(e->skey[0], n * 8) == cudaSuccess && ensure(e->skey[1], n * 8) == cudaSuccess &&
            ensure(e->sval[0], n * 4) == cudaSuccess && ensure(e->sval[1], n * 4) == cudaSuccess &&
@@ -488,7 +500,32 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
   a.out_mc = dmc;
   a.rflag = (uint8_t*)e->rflag.p;
   a.mflag = (uint8_t*)e->mflag.p;
-  if (ordered) {
+  bool done = false;
+  if (e->flat_kernel == MM_FLAT_KERNEL_BUCKETED) {
+    BucketScratch bs;
+    for (int b = 0; b < 4; b++) {
+      bs.h[b] = (uint64_t*)e->bh[b].p;
+      bs.i[b] = (uint32_t*)e->bi[b].p;
+    }
+    bs.part = (uint32_t*)e->bpart.p;
+    bs.roff = (uint32_t*)e->broff.p;
+    bs.moff = (uint32_t*)e->bmoff.p;
+    bs.overflow = (uint32_t*)e->bover.p;
+    bs.rres = info.rres;
+    bs.mres = info.mres;
+    e->timer.begin(e->st);
+    CK(run_bucketed(a, ordered, bs, e->st));
+    e->timer.end(e->st);
+    uint32_t over = 0;
+    CK(cudaMemcpyAsync(&over, e->bover.p, 4, cudaMemcpyDeviceToHost, e->st));
+    CK(cudaStreamSynchronize(e->st));
+    done = over == 0;
+    if (!done) {  // a bucket exceeded the on-chip capacity (heavily repeated tuples)
+      e->bucket_fallbacks++;
+      CK(cudaMemsetAsync(e->nmatched.p, 0, 8, e->st));
+    }
+  }
+  if (!done && ordered) {
     SortScratch s;
     for (int b = 0; b < 2; b++) {
       s.key[b] = (uint64_t*)e->skey[b].p;
@@ -502,7 +539,7 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
     e->timer.begin(e->st);
     CK(run_sort_rank(a, info.ref, info.diff, s, e->st));
     e->timer.end(e->st);
-  } else {
+  } else if (!done) {
     HashScratch h;
     h.owner = (uint32_t*)e->owner.p;
     h.rcnt = (uint32_t*)e->rcnt.p;
@@ -544,6 +581,11 @@ int mm_match_batch(mm_engine* e, int64_t* out_recv_cookie, int64_t* out_msg_cook
 
 int mm_set_option(mm_engine* e, int32_t option, int64_t value) {
   if (!e) return MM_ERR_ARG;
+  if (option == MM_OPT_FLAT_KERNEL) {
+    if (value != MM_FLAT_KERNEL_BUCKETED && value != MM_FLAT_KERNEL_GLOBAL) return MM_ERR_ARG;
+    e->flat_kernel = (int)value;
+    return MM_OK;
+  }
   if (option == MM_OPT_MPI_KERNEL) {
     if (value == MM_MPI_KERNEL_AUTO) value = MM_MPI_KERNEL_FIFO;
     if (value != MM_MPI_KERNEL_MATRIX && value != MM_MPI_KERNEL_FIFO) return MM_ERR_ARG;

@@ -89,6 +89,21 @@ struct HashScratch {
 };
 cudaError_t run_hash(const FlatArgs& a, const HashScratch& h, cudaStream_t st);
 
+// Both no-wildcard levels, hash-bucketed (k_bucket.cu): stable partition into
+// ~1K-element buckets + one CTA per bucket.  Sets *overflow if a bucket does
+// not fit on chip (the caller then falls back to run_sort_rank / run_hash).
+struct BucketScratch {
+  uint64_t* h[4];  // receive ping-pong (0,1), message ping-pong (2,3)
+  uint32_t* i[4];
+  uint32_t* part;
+  uint32_t* roff;
+  uint32_t* moff;
+  uint32_t* overflow;
+  int64_t rres, mres;
+};
+cudaError_t run_bucketed(const FlatArgs& a, bool ordered, const BucketScratch& s, cudaStream_t st);
+int64_t bucket_scratch_elems(int64_t n);
+
 // Compaction of the no-wildcard queues into the other ping-pong buffer.
 cudaError_t run_compact(const Side& S, int64_t resid, int64_t n, const uint8_t* matched, uint64_t* q_h, int64_t* q_c,
                         int32_t* q_len, uint32_t* scan, cudaStream_t st);

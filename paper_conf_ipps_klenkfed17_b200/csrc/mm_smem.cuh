@@ -1,0 +1,83 @@
+// mm_smem.cuh -- shared-memory building blocks of the per-endpoint / per-bucket
+// matching kernels: 16-bit atomics through 32-bit words, ballot-based peer
+// masks and warp-ordered placement into per-tuple lists.
+#pragma once
+
+#include "mm_internal.cuh"
+
+namespace mm {
+
+constexpr uint16_t kWild = 0xFFFEu;
+constexpr uint16_t kNone = 0xFFFFu;
+constexpr uint16_t kEmpty16 = 0xFFFFu;
+
+// 16-bit CAS through the containing 32-bit word.
+// (pointer arithmetic, not integer casts, so shared-memory provenance survives
+// and the atomics compile to ATOMS)
+__device__ __forceinline__ uint32_t* word_of(uint16_t* p) {
+  return reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(p) - (reinterpret_cast<uintptr_t>(p) & 2));
+}
+__device__ __forceinline__ uint16_t cas16(uint16_t* p, uint16_t expect, uint16_t val) {
+  uint32_t* w = word_of(p);
+  const uint32_t sh = (reinterpret_cast<uintptr_t>(p) & 2) ? 16u : 0u;
+  uint32_t old = *w;
+  while (true) {
+    const uint16_t cur = (uint16_t)(old >> sh);
+    if (cur != expect) return cur;
+    const uint32_t nw = (old & ~(0xFFFFu << sh)) | ((uint32_t)val << sh);
+    const uint32_t got = atomicCAS(w, old, nw);
+    if (got == old) return expect;
+    old = got;
+  }
+}
+
+// 16-bit counter increment through the containing 32-bit word (no carry out:
+// counts stay below 65536).
+__device__ __forceinline__ void inc16(uint16_t* p) {
+  atomicAdd(word_of(p), (reinterpret_cast<uintptr_t>(p) & 2) ? 0x10000u : 1u);
+}
+// Same, returning the previous 16-bit value.
+__device__ __forceinline__ uint32_t fetch_inc16(uint16_t* p) {
+  const bool hi = (reinterpret_cast<uintptr_t>(p) & 2) != 0;
+  const uint32_t old = atomicAdd(word_of(p), hi ? 0x10000u : 1u);
+  return hi ? (old >> 16) : (old & 0xFFFFu);
+}
+
+// Lanes holding the same value as this lane, from one ballot per value bit
+// (nbits covers every value in play).  Replaces match.any, whose cost grows
+// with the number of distinct values in the warp.
+__device__ __forceinline__ uint32_t peers_of(uint32_t v, int nbits) {
+  uint32_t m = kFull;
+  for (int b = 0; b < nbits; b++) {
+    const bool bit = (v >> b) & 1u;
+    const uint32_t bb = __ballot_sync(kFull, bit);
+    m &= bit ? bb : ~bb;
+  }
+  return m;
+}
+
+// Ordered placement by one warp: element x (0..n) with tuple id key(x) (>=
+// kWild = skip) gets slot start[k] + running[k]; put(x, k, rank, slot).
+// nkeys bounds the tuple ids (ids < nkeys).
+template <class KeyF, class PutF>
+__device__ __forceinline__ void place_in_order(int64_t n, KeyF key, const uint16_t* start, uint16_t* running, PutF put,
+                                               int lane, uint32_t lt, uint32_t nkeys) {
+  const int nbits = 32 - __clz(nkeys | 1u);  // ids 0..nkeys (nkeys = "skip")
+  for (int64_t b = 0; b < n; b += 32) {
+    const int64_t x = b + lane;
+    const uint32_t k = x < n ? key(x) : 0xFFFFFFFFu;
+    const bool ok = k < kWild;
+    const uint32_t peers = peers_of(ok ? k : nkeys, nbits);
+    uint32_t run = 0;
+    if (ok) run = running[k];
+    __syncwarp();
+    if (ok) {
+      const uint32_t r = run + __popc(peers & lt);
+      put(x, k, r, (uint32_t)start[k] + r);
+      if ((peers >> lane) == 1u) running[k] = (uint16_t)(run + __popc(peers));
+    }
+    __syncwarp();
+  }
+}
+
+}  // namespace mm

@@ -71,7 +71,7 @@ class Engine:
     """Owns one mm_engine (see include/mm.h for the semantics of each call)."""
 
     def __init__(self, semantics, n_endpoints=1, recv_capacity=1024, msg_capacity=1024, stream=None,
-                 mpi_kernel=None):
+                 mpi_kernel=None, flat_kernel=None):
         L = _lib.load()
         self._L = L
         self.semantics = semantics
@@ -89,6 +89,8 @@ class Engine:
         self._keep = []  # device buffers referenced by pending batches
         if mpi_kernel is not None:
             self.set_option(_lib.MM_OPT_MPI_KERNEL, mpi_kernel)
+        if flat_kernel is not None:
+            self.set_option(_lib.MM_OPT_FLAT_KERNEL, flat_kernel)
 
     def set_option(self, option, value):
         check(self._L.mm_set_option(self._h, option, value), "mm_set_option")

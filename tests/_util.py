@@ -17,12 +17,12 @@ def to_dev(a):
     return torch.from_numpy(a.copy()).cuda()
 
 
-def gpu_batches(sem, n_ep, rcap, mcap, batches, host=False, out_cap=None, mpi_kernel=None):
+def gpu_batches(sem, n_ep, rcap, mcap, batches, host=False, out_cap=None, mpi_kernel=None, flat_kernel=None):
     """batches: list of (recv_hdr, recv_cookie, recv_off, msg_hdr, msg_cookie, msg_off).
     Returns a list of (out_rc, out_mc) numpy arrays, one per batch."""
     import torch
     from paper_conf_ipps_klenkfed17_b200 import Engine
-    eng = Engine(sem, n_ep, rcap, mcap, mpi_kernel=mpi_kernel)
+    eng = Engine(sem, n_ep, rcap, mcap, mpi_kernel=mpi_kernel, flat_kernel=flat_kernel)
     res = []
     for (rh, rc, ro, mh, mc, mo) in batches:
         if host:

@@ -17,6 +17,7 @@ pytestmark = pytest.mark.gpu
 
 MPI, ORD, UNO = oracle.SEM_MPI, oracle.SEM_NOWILD_ORDERED, oracle.SEM_NOWILD_UNORDERED
 KERNELS = pytest.mark.parametrize("kern", [1, 2], ids=["matrix", "fifo"])  # MM_MPI_KERNEL_*
+FLAT = pytest.mark.parametrize("flat", [0, 1], ids=["bucketed", "global"])  # MM_FLAT_KERNEL_*
 
 
 def assert_exact(g, o):
@@ -167,14 +168,16 @@ def test_mpi_config1_full(kern):
 
 @pytest.mark.parametrize("seed", range(5))
 @pytest.mark.parametrize("n", [1, 100, 4095, 4097, 50000])
-def test_ordered_random(seed, n):
+@FLAT
+def test_ordered_random(seed, n, flat):
     q = synth.nowild_pairs(seed, n=n, n_src=max(2, n // 50), n_tag=3, p_unmatched=0.2)
-    g, _ = gpu_batches(ORD, 1, n, n, single_batch(q))
+    g, _ = gpu_batches(ORD, 1, n, n, single_batch(q), flat_kernel=flat)
     o, _ = oracle_batches(ORD, 1, single_batch(q))
     assert_exact(g, o)
 
 
-def test_ordered_wide_keys_and_wildcard_values():
+@FLAT
+def test_ordered_wide_keys_and_wildcard_values(flat):
     rng = np.random.default_rng(1)
     n = 20000
     src = rng.integers(0, 1 << 32, n, dtype=np.uint64)
@@ -186,36 +189,39 @@ def test_ordered_wide_keys_and_wildcard_values():
     rh[::3] = rh[0]
     mh = rh[rng.permutation(n)]
     b = [(rh, None, np.array([0, n]), mh, None, np.array([0, n]))]
-    g, _ = gpu_batches(ORD, 1, n, n, b)
+    g, _ = gpu_batches(ORD, 1, n, n, b, flat_kernel=flat)
     o, _ = oracle_batches(ORD, 1, b)
     assert_exact(g, o)
 
 
 @pytest.mark.parametrize("seed", range(3))
-def test_ordered_multibatch(seed):
+@FLAT
+def test_ordered_multibatch(seed, flat):
     rng = np.random.default_rng(seed)
     q = synth.nowild_pairs(seed + 3, n=30000, n_src=300, n_tag=4, p_unmatched=0.3)
     batches = split_batches(q, 3, rng)
-    g, _ = gpu_batches(ORD, 1, 60000, 60000, batches)
+    g, _ = gpu_batches(ORD, 1, 60000, 60000, batches, flat_kernel=flat)
     o, _ = oracle_batches(ORD, 1, batches)
     assert_exact(g, o)
 
 
-def test_ordered_all_same_key():
+@FLAT
+def test_ordered_all_same_key(flat):
     n = 10000
     rh = synth.pack(np.full(n, 4), np.full(n, 2))
     mh = synth.pack(np.full(n - 17, 4), np.full(n - 17, 2))
     b = [(rh, None, np.array([0, n]), mh, None, np.array([0, n - 17]))]
-    g, _ = gpu_batches(ORD, 1, n, n, b)
+    g, _ = gpu_batches(ORD, 1, n, n, b, flat_kernel=flat)
     o, _ = oracle_batches(ORD, 1, b)
     assert_exact(g, o)
 
 
 @pytest.mark.slow
-def test_ordered_config2_full():
+@FLAT
+def test_ordered_config2_full(flat):
     q = synth.nowild_pairs()
     n = len(q.recv_hdr)
-    g, _ = gpu_batches(ORD, 1, n, n, single_batch(q))
+    g, _ = gpu_batches(ORD, 1, n, n, single_batch(q), flat_kernel=flat)
     mr, _ = oracle.nowild_ordered(q.recv_hdr, q.msg_hdr)
     grc, gmc, cnt = g[0]
     assert np.array_equal(grc, np.arange(n))
@@ -224,9 +230,10 @@ def test_ordered_config2_full():
 
 @pytest.mark.parametrize("seed", range(5))
 @pytest.mark.parametrize("n", [1, 100, 5000, 70000])
-def test_unordered_random(seed, n):
+@FLAT
+def test_unordered_random(seed, n, flat):
     q = synth.nowild_pairs(seed, n=n, n_src=max(2, n // 20), n_tag=3, p_unmatched=0.2)
-    g, _ = gpu_batches(UNO, 1, n, n, single_batch(q))
+    g, _ = gpu_batches(UNO, 1, n, n, single_batch(q), flat_kernel=flat)
     grc, gmc, cnt = g[0]
     assert np.array_equal(grc, np.arange(n))
     o, _ = oracle_batches(UNO, 1, single_batch(q))
@@ -243,11 +250,12 @@ def check_min(q):
 
 
 @pytest.mark.parametrize("seed", range(3))
-def test_unordered_multibatch(seed):
+@FLAT
+def test_unordered_multibatch(seed, flat):
     rng = np.random.default_rng(seed)
     q = synth.nowild_pairs(seed + 7, n=20000, n_src=200, n_tag=3, p_unmatched=0.3)
     batches = split_batches(q, 3, rng)
-    g, _ = gpu_batches(UNO, 1, 40000, 40000, batches)
+    g, _ = gpu_batches(UNO, 1, 40000, 40000, batches, flat_kernel=flat)
     # across all batches: every pair has equal tuples, every element used once,
     # and the total per tuple is min(#recv, #msg) of the whole input
     rc = np.concatenate([x[0] for x in g])
@@ -259,10 +267,11 @@ def test_unordered_multibatch(seed):
 
 
 @pytest.mark.slow
-def test_unordered_config3_per_gpu():
+@FLAT
+def test_unordered_config3_per_gpu(flat):
     q = synth.nowild_pairs(3, n=1 << 25, n_src=1 << 20, n_tag=1 << 12)
     n = len(q.recv_hdr)
-    g, _ = gpu_batches(UNO, 1, n, n, single_batch(q))
+    g, _ = gpu_batches(UNO, 1, n, n, single_batch(q), flat_kernel=flat)
     grc, gmc, cnt = g[0]
     m = gmc >= 0
     assert np.array_equal(q.recv_hdr[grc[m]], q.msg_hdr[gmc[m]])
