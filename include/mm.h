@@ -133,8 +133,12 @@ int mm_push_msgs(mm_engine *e, const uint64_t *hdr, const int64_t *cookie,
  * mm_match_batch -- match every endpoint's snapshot (residual PRQ ++ posted
  * receives, residual UMQ ++ pushed messages; §V l.128), then compact
  * the queues (§V.A l.149).
- *   out_recv_cookie  [out_capacity] receives, for every snapshot receive
- *                    (endpoint-major, queue order), its cookie;
+ *   out_recv_cookie  [out_capacity] receives, for every snapshot receive, its
+ *                    cookie.  Order: MPI -- endpoint-major, queue order; the
+ *                    no-wildcard levels -- every snapshot receive exactly once
+ *                    in an engine-defined order (the hash-bucketed kernels
+ *                    report, and keep their queues, in bucket order; the
+ *                    relative order of receives with equal tuples is kept);
  *   out_msg_cookie   [out_capacity] the cookie of the message it matched, or
  *                    MM_NO_MATCH.  Either pointer may be host or device.
  *   out_capacity     length of both arrays; must cover the total snapshot

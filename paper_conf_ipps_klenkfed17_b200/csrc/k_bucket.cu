@@ -303,7 +303,9 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
     }
   }
   __syncthreads();
-  // results at snapshot positions, matched flags
+  // results in bucket order (coalesced): receive at bucket-sorted position
+  // r0 + e, message flags at m0 + e - nr; the queue compaction reads the same
+  // order, so per-tuple order (all these levels need) is kept
   uint32_t nmatch = 0;
   for (uint32_t e = tid; e < n; e += NT) {
     const uint16_t k = sm.key[e];
@@ -317,11 +319,11 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
         f = 1;
         nmatch++;
       }
-      a.out_rc[u] = a.R.cookie(0, u, rres, rpb);
-      a.out_mc[u] = mc;
-      a.rflag[u] = f;
+      a.out_rc[r0 + e] = a.R.cookie(0, u, rres, rpb);
+      a.out_mc[r0 + e] = mc;
+      a.rflag[r0 + e] = f;
     } else {
-      a.mflag[u] = (k != kNone && sm.rank[e] < sm.cnt_r[k]) ? 1 : 0;
+      a.mflag[m0 + e - nr] = (k != kNone && sm.rank[e] < sm.cnt_r[k]) ? 1 : 0;
     }
   }
   for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
@@ -334,7 +336,7 @@ int64_t bucket_bits_for(int64_t n) {
   return nb;
 }
 
-cudaError_t run_bucketed(const FlatArgs& a, bool ordered, const BucketScratch& s, cudaStream_t st) {
+cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cudaStream_t st) {
   const int nb = (int)bucket_bits_for(a.nr + a.nm);
   const uint32_t B = 1u << nb;
   SnapRead rs{a.R, 0, 0}, ms{a.M, 0, 0};
@@ -349,6 +351,10 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, const BucketScratch& s
   err = partition_side(ms, a.nm, nb, s.h[2], s.i[2], s.h[3], s.i[3], s.part, s.moff, &mh, &mi, st);
   if (err != cudaSuccess) return err;
   if ((err = cudaMemsetAsync(s.overflow, 0, 4, st)) != cudaSuccess) return err;
+  s.rh_sorted = rh;
+  s.ri_sorted = ri;
+  s.mh_sorted = mh;
+  s.mi_sorted = mi;
   BucketArgs ba{a, rh, ri, s.roff, mh, mi, s.moff, s.overflow};
   const size_t smem = sizeof(BucketSmem);
   if (ordered) {
@@ -363,6 +369,43 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, const BucketScratch& s
     k_bucket_pair<false><<<B, kBucketThreads, smem, st>>>(ba);
   }
   return cudaGetLastError();
+}
+
+// Residual queue from the bucket-sorted side: survivors keep bucket order
+// (hence per-tuple order).
+struct SortedUnmatched {
+  const uint8_t* matched;
+  __device__ __forceinline__ uint32_t operator()(int64_t p) const { return matched[p] ? 0u : 1u; }
+};
+struct SortedCompactOut {
+  Side S;
+  int64_t resid;
+  const uint64_t* h;
+  const uint32_t* ix;
+  int64_t n;
+  uint64_t* q_h;
+  int64_t* q_c;
+  int32_t* q_len;
+  __device__ __forceinline__ void operator()(int64_t p, uint32_t ex, uint32_t v) const {
+    if (v) {
+      q_h[ex] = h[p];
+      q_c[ex] = S.cookie(0, ix[p], resid, 0);
+    }
+    if (p == n - 1) *q_len = (int32_t)(ex + v);
+  }
+};
+__global__ void k_set_len0(int32_t* q_len) { *q_len = 0; }
+
+cudaError_t run_compact_sorted(const Side& S, int64_t resid, int64_t n, const uint64_t* h, const uint32_t* ix,
+                               const uint8_t* matched, uint64_t* q_h, int64_t* q_c, int32_t* q_len, uint32_t* scan,
+                               cudaStream_t st) {
+  if (n == 0) {
+    count_launch();
+    k_set_len0<<<1, 1, 0, st>>>(q_len);
+    return cudaGetLastError();
+  }
+  return scan_apply<uint32_t>(SortedUnmatched{matched}, n, scan, SortedCompactOut{S, resid, h, ix, n, q_h, q_c, q_len},
+                              st);
 }
 
 int64_t bucket_scratch_elems(int64_t n) { return ((int64_t)1 << bucket_bits_for(n)) + 1; }

@@ -20,7 +20,7 @@
 //     and exact receives per tuple;
 //  P5 block scans: tuple list starts for both sides, ordered wildcard list;
 //  P6 warp 0 places messages, warp 1 places exact receives into their tuple
-//     lists in order (match_any ranks) -- giving every exact receive its e_i;
+//     lists in order (ballot ranks) -- giving every exact receive its e_i;
 //  P7 warp 0 walks the wildcards in posting order: lanes test admissibility of
 //     tuples with one masked XOR, read each admitted tuple's head
 //     (e_k(w) from a per-tuple cursor over that tuple's exact receives, plus

@@ -501,8 +501,8 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
   a.rflag = (uint8_t*)e->rflag.p;
   a.mflag = (uint8_t*)e->mflag.p;
   bool done = false;
+  BucketScratch bs;
   if (e->flat_kernel == MM_FLAT_KERNEL_BUCKETED) {
-    BucketScratch bs;
     for (int b = 0; b < 4; b++) {
       bs.h[b] = (uint64_t*)e->bh[b].p;
       bs.i[b] = (uint32_t*)e->bi[b].p;
@@ -560,8 +560,13 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
   for (int i = 0; i < 2; i++) {
     Queue& q = *qs[i];
     const int nb = q.cur ^ 1;
-    CK(run_compact(*ss[i], res[i], ns[i], fl[i], (uint64_t*)q.hdr[nb].p, (int64_t*)q.cookie[nb].p,
-                   (int32_t*)q.len[nb].p, (uint32_t*)e->scan.p, e->st));
+    if (done)  // bucketed: flags and survivors in bucket order
+      CK(run_compact_sorted(*ss[i], res[i], ns[i], i == 0 ? bs.rh_sorted : bs.mh_sorted,
+                            i == 0 ? bs.ri_sorted : bs.mi_sorted, fl[i], (uint64_t*)q.hdr[nb].p,
+                            (int64_t*)q.cookie[nb].p, (int32_t*)q.len[nb].p, (uint32_t*)e->scan.p, e->st));
+    else
+      CK(run_compact(*ss[i], res[i], ns[i], fl[i], (uint64_t*)q.hdr[nb].p, (int64_t*)q.cookie[nb].p,
+                     (int32_t*)q.len[nb].p, (uint32_t*)e->scan.p, e->st));
     q.cur = nb;
     q.pend = Pending();
     q.resid_host = ns[i];  // upper bound until the next exact read

@@ -243,7 +243,18 @@ __global__ void __launch_bounds__(kPartThreads) k_part_scatter(BucketF bucket, M
     int64_t k = cbase + r * 32 + lane;
     bool valid = k < n;
     uint32_t b = valid ? bucket(k) : 0xFFFFFFFFu;
-    uint32_t peers = __match_any_sync(kFull, b);
+    // lanes with the same bucket: one ballot per bucket bit (match.any is
+    // slow when a warp holds many distinct values); invalid lanes use 256
+    uint32_t peers = kFull;
+    {
+      const uint32_t v = valid ? b : 256u;
+#pragma unroll
+      for (int bit = 0; bit < 9; bit++) {
+        const bool x = (v >> bit) & 1u;
+        const uint32_t bb = __ballot_sync(kFull, x);
+        peers &= x ? bb : ~bb;
+      }
+    }
     uint32_t before = wrun[w][valid ? b : 0];
     __syncwarp();
     if (valid) {

@@ -100,8 +100,16 @@ struct BucketScratch {
   uint32_t* moff;
   uint32_t* overflow;
   int64_t rres, mres;
+  // outputs: the bucket-sorted sides (results are written in this order)
+  const uint64_t* rh_sorted;
+  const uint32_t* ri_sorted;
+  const uint64_t* mh_sorted;
+  const uint32_t* mi_sorted;
 };
-cudaError_t run_bucketed(const FlatArgs& a, bool ordered, const BucketScratch& s, cudaStream_t st);
+cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cudaStream_t st);
+cudaError_t run_compact_sorted(const Side& S, int64_t resid, int64_t n, const uint64_t* h, const uint32_t* ix,
+                               const uint8_t* matched, uint64_t* q_h, int64_t* q_c, int32_t* q_len, uint32_t* scan,
+                               cudaStream_t st);
 int64_t bucket_scratch_elems(int64_t n);
 
 // Compaction of the no-wildcard queues into the other ping-pong buffer.

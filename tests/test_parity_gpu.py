@@ -32,6 +32,23 @@ def assert_exact(g, o):
 
 
 @KERNELS
+def assert_same_pairs(g, o):
+    """No-wildcard levels report receives in an engine-defined order: compare
+    the receive->message map per batch (bit-exact as a map)."""
+    assert len(g) == len(o)
+    for b, ((grc, gmc, cnt), (orc, omc)) in enumerate(zip(g, o)):
+        assert len(grc) == len(orc), "batch %d: snapshot sizes differ" % b
+        assert len(np.unique(grc)) == len(grc), "batch %d: a receive reported twice" % b
+        gm = dict(zip(grc.tolist(), gmc.tolist()))
+        om = dict(zip(orc.tolist(), omc.tolist()))
+        assert set(gm) == set(om), "batch %d: different receives" % b
+        bad = [k for k in om if gm[k] != om[k]]
+        assert not bad, "batch %d: %d mismatches, e.g. recv %s: gpu %s oracle %s" % (
+            b, len(bad), bad[0], gm[bad[0]], om[bad[0]])
+        assert int(cnt[1]) == int((omc >= 0).sum())
+
+
+@KERNELS
 def test_mpi_config0(kern):
     q = synth.mpi_small(0)
     g, _ = gpu_batches(MPI, 1, 64, 64, single_batch(q), mpi_kernel=kern)
@@ -173,7 +190,7 @@ def test_ordered_random(seed, n, flat):
     q = synth.nowild_pairs(seed, n=n, n_src=max(2, n // 50), n_tag=3, p_unmatched=0.2)
     g, _ = gpu_batches(ORD, 1, n, n, single_batch(q), flat_kernel=flat)
     o, _ = oracle_batches(ORD, 1, single_batch(q))
-    assert_exact(g, o)
+    assert_same_pairs(g, o)
 
 
 @FLAT
@@ -191,7 +208,7 @@ def test_ordered_wide_keys_and_wildcard_values(flat):
     b = [(rh, None, np.array([0, n]), mh, None, np.array([0, n]))]
     g, _ = gpu_batches(ORD, 1, n, n, b, flat_kernel=flat)
     o, _ = oracle_batches(ORD, 1, b)
-    assert_exact(g, o)
+    assert_same_pairs(g, o)
 
 
 @pytest.mark.parametrize("seed", range(3))
@@ -202,7 +219,7 @@ def test_ordered_multibatch(seed, flat):
     batches = split_batches(q, 3, rng)
     g, _ = gpu_batches(ORD, 1, 60000, 60000, batches, flat_kernel=flat)
     o, _ = oracle_batches(ORD, 1, batches)
-    assert_exact(g, o)
+    assert_same_pairs(g, o)
 
 
 @FLAT
@@ -213,7 +230,7 @@ def test_ordered_all_same_key(flat):
     b = [(rh, None, np.array([0, n]), mh, None, np.array([0, n - 17]))]
     g, _ = gpu_batches(ORD, 1, n, n, b, flat_kernel=flat)
     o, _ = oracle_batches(ORD, 1, b)
-    assert_exact(g, o)
+    assert_same_pairs(g, o)
 
 
 @pytest.mark.slow
@@ -224,8 +241,10 @@ def test_ordered_config2_full(flat):
     g, _ = gpu_batches(ORD, 1, n, n, single_batch(q), flat_kernel=flat)
     mr, _ = oracle.nowild_ordered(q.recv_hdr, q.msg_hdr)
     grc, gmc, cnt = g[0]
-    assert np.array_equal(grc, np.arange(n))
-    assert np.array_equal(gmc, mr), "mismatches: %d" % int((gmc != mr).sum())
+    assert np.array_equal(np.sort(grc), np.arange(n))
+    got = np.empty(n, np.int64)
+    got[grc] = gmc
+    assert np.array_equal(got, mr), "mismatches: %d" % int((got != mr).sum())
 
 
 @pytest.mark.parametrize("seed", range(5))
@@ -235,7 +254,7 @@ def test_unordered_random(seed, n, flat):
     q = synth.nowild_pairs(seed, n=n, n_src=max(2, n // 20), n_tag=3, p_unmatched=0.2)
     g, _ = gpu_batches(UNO, 1, n, n, single_batch(q), flat_kernel=flat)
     grc, gmc, cnt = g[0]
-    assert np.array_equal(grc, np.arange(n))
+    assert np.array_equal(np.sort(grc), np.arange(n))
     o, _ = oracle_batches(UNO, 1, single_batch(q))
     # per-tuple counts are unique: compare them with the oracle's result
     orc, omc = o[0]
