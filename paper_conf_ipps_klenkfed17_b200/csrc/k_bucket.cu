@@ -57,9 +57,13 @@ struct BMove {
   const uint32_t* ix;
   uint64_t* oh;
   uint32_t* oi;
-  __device__ __forceinline__ void operator()(int64_t k, int64_t dst) const {
-    oh[dst] = FIRST ? snap.hdr(k) : h[k];
-    oi[dst] = FIRST ? (uint32_t)k : ix[k];
+  __device__ __forceinline__ void load(int64_t k, uint64_t& a, uint64_t& b) const {
+    a = FIRST ? snap.hdr(k) : h[k];
+    b = FIRST ? (uint64_t)k : ix[k];
+  }
+  __device__ __forceinline__ void store(int64_t dst, uint64_t a, uint64_t b) const {
+    oh[dst] = a;
+    oi[dst] = (uint32_t)b;
   }
 };
 
@@ -140,6 +144,7 @@ struct BucketArgs {
   uint32_t* overflow;
 };
 
+template <bool ORDERED>
 struct BucketSmem {
   uint64_t hdr[kBucketCap];      // receives [0, nr), then messages [nr, nr + nm)
   uint32_t idx[kBucketCap];      // snapshot index
@@ -151,7 +156,7 @@ struct BucketSmem {
   uint16_t start_m[kBucketCap];  // start of the tuple in by_key
   uint16_t cnt_r[kBucketCap];    // receives per tuple
   uint16_t by_key[kBucketCap];   // messages grouped by tuple, in rank order (element index)
-  uint16_t pcnt[8][kBucketCap];  // per-quarter counts / running ranks
+  uint16_t pcnt[ORDERED ? 8 : 2][kBucketCap];  // per-quarter counts / running ranks (msgs, then receives)
   uint32_t scan[kBucketThreads / 32 + 1];
   uint32_t K;
   uint32_t matched;
@@ -160,7 +165,8 @@ struct BucketSmem {
 template <bool ORDERED>
 __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
-  BucketSmem& sm = *reinterpret_cast<BucketSmem*>(smem_raw);
+  BucketSmem<ORDERED>& sm = *reinterpret_cast<BucketSmem<ORDERED>*>(smem_raw);
+  constexpr int RROW = ORDERED ? 4 : 1;  // first pcnt row of the receive side
   constexpr int NT = kBucketThreads;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t lt = lanemask_lt();
@@ -216,7 +222,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
       if (sm.table[s] != kEmpty16) {
         sm.slot_id[s] = (uint16_t)id;
 #pragma unroll
-        for (int q = 0; q < 8; q++) sm.pcnt[q][id] = 0;
+        for (int q = 0; q < (ORDERED ? 8 : 2); q++) sm.pcnt[q][id] = 0;
         id++;
       }
     if (tid == 0) sm.K = tot;
@@ -247,7 +253,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
     if (k != kNone) {
       const uint32_t side_n = is_msg ? nm : nr, x = is_msg ? e - nr : e;
       const uint32_t q = ORDERED ? (uint32_t)(((uint64_t)x * 4) / side_n) : 0u;
-      inc16(&sm.pcnt[(is_msg ? 0 : 4) + q][k]);
+      inc16(&sm.pcnt[(is_msg ? 0 : RROW) + q][k]);
     }
   }
   __syncthreads();
@@ -259,9 +265,9 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
       uint32_t rm = 0, rr = 0;
 #pragma unroll
       for (int q = 0; q < (ORDERED ? 4 : 1); q++) {
-        const uint32_t x = sm.pcnt[q][k], y = sm.pcnt[4 + q][k];
+        const uint32_t x = sm.pcnt[q][k], y = sm.pcnt[RROW + q][k];
         sm.pcnt[q][k] = (uint16_t)rm;
-        sm.pcnt[4 + q][k] = (uint16_t)rr;
+        sm.pcnt[RROW + q][k] = (uint16_t)rr;
         rm += x;
         rr += y;
       }
@@ -285,7 +291,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
     const int64_t x0 = ((int64_t)side_n * q + 3) / 4, x1 = ((int64_t)side_n * (q + 1) + 3) / 4;
     place_in_order(
         x1 - x0, [&](int64_t x) { return (uint32_t)sm.key[base + x0 + x]; }, msg_side ? sm.start_m : sm.start_m,
-        sm.pcnt[warp],
+        sm.pcnt[ORDERED ? warp : 0],
         [&](int64_t x, uint32_t k, uint32_t r, uint32_t slot) {
           const uint32_t e = base + (uint32_t)(x0 + x);
           sm.rank[e] = (uint16_t)r;
@@ -297,7 +303,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
       const uint16_t k = sm.key[e];
       if (k == kNone) continue;
       const bool is_msg = e >= nr;
-      const uint32_t r = fetch_inc16(&sm.pcnt[is_msg ? 0 : 4][k]);
+      const uint32_t r = fetch_inc16(&sm.pcnt[is_msg ? 0 : RROW][k]);
       sm.rank[e] = (uint16_t)r;
       if (is_msg) sm.by_key[sm.start_m[k] + r] = (uint16_t)e;
     }
@@ -356,13 +362,14 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cuda
   s.mh_sorted = mh;
   s.mi_sorted = mi;
   BucketArgs ba{a, rh, ri, s.roff, mh, mi, s.moff, s.overflow};
-  const size_t smem = sizeof(BucketSmem);
   if (ordered) {
+    const size_t smem = sizeof(BucketSmem<true>);
     err = cudaFuncSetAttribute(k_bucket_pair<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (err != cudaSuccess) return err;
     count_launch();
     k_bucket_pair<true><<<B, kBucketThreads, smem, st>>>(ba);
   } else {
+    const size_t smem = sizeof(BucketSmem<false>);
     err = cudaFuncSetAttribute(k_bucket_pair<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (err != cudaSuccess) return err;
     count_launch();

@@ -99,9 +99,13 @@ struct MoveKV {
   const uint32_t* vi;
   uint64_t* ko;
   uint32_t* vo;
-  __device__ __forceinline__ void operator()(int64_t k, int64_t dst) const {
-    ko[dst] = ki[k];
-    vo[dst] = vi[k];
+  __device__ __forceinline__ void load(int64_t k, uint64_t& a, uint64_t& b) const {
+    a = ki[k];
+    b = vi[k];
+  }
+  __device__ __forceinline__ void store(int64_t dst, uint64_t a, uint64_t b) const {
+    ko[dst] = a;
+    vo[dst] = (uint32_t)b;
   }
 };
 
@@ -398,9 +402,13 @@ struct MoveRoute {
   uint64_t* oa;
   int64_t* ob;
   int64_t base;
-  __device__ __forceinline__ void operator()(int64_t k, int64_t dst) const {
-    oa[dst] = a[k];
-    ob[dst] = b ? b[k] : (base + k);
+  __device__ __forceinline__ void load(int64_t k, uint64_t& x, uint64_t& y) const {
+    x = a[k];
+    y = (uint64_t)(b ? b[k] : (base + k));
+  }
+  __device__ __forceinline__ void store(int64_t dst, uint64_t x, uint64_t y) const {
+    oa[dst] = x;
+    ob[dst] = (int64_t)y;
   }
 };
 __global__ void k_route_counts(const uint32_t* hist, int64_t ntiles, int world, int64_t n, int64_t* counts) {

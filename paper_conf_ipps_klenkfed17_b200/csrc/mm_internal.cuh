@@ -224,25 +224,43 @@ __global__ void __launch_bounds__(kPartThreads) k_part_hist(BucketF bucket, int6
 }
 
 // Scatter: element k of bucket b goes to off[b * ntiles + tile] + its rank
-// among the tile's bucket-b elements in input order.  move(k, dst) performs
-// the data movement.
+// among the tile's bucket-b elements in input order.  The payload moves
+// through shared memory: elements are first placed in tile-local bucket order,
+// then written out so that consecutive threads write consecutive addresses of
+// a bucket's run (coalesced stores instead of one scattered store per lane).
+// move.load(k, a, b) reads element k's payload, move.store(dst, a, b) writes it.
+constexpr size_t kPartSmem = (size_t)kPartTile * (8 + 8 + 2) + (kPartWarps + 3) * 256 * 4 + 64;
+
 template <class BucketF, class MoveF>
 __global__ void __launch_bounds__(kPartThreads) k_part_scatter(BucketF bucket, MoveF move, int64_t n, int nbuckets,
                                                                int64_t ntiles, const uint32_t* off) {
-  __shared__ uint32_t wrun[kPartWarps][256];
-  __shared__ uint32_t base_s[256];
+  extern __shared__ __align__(16) uint8_t part_smem[];
+  uint64_t* sa = reinterpret_cast<uint64_t*>(part_smem);
+  uint64_t* sb = sa + kPartTile;
+  uint32_t* wrun = reinterpret_cast<uint32_t*>(sb + kPartTile);  // [kPartWarps][256]
+  uint32_t* lstart = wrun + kPartWarps * 256;                     // tile-local bucket starts
+  uint32_t* gbase = lstart + 256;                                 // global bucket bases
+  uint32_t* scan_sm = gbase + 256;
+  uint16_t* sbk = reinterpret_cast<uint16_t*>(scan_sm + 64);
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  for (int b = lane; b < 256; b += 32) wrun[w][b] = 0;
-  for (int b = threadIdx.x; b < nbuckets; b += blockDim.x) base_s[b] = off[(int64_t)b * ntiles + blockIdx.x];
+  for (int b = lane; b < 256; b += 32) wrun[w * 256 + b] = 0;
+  for (int b = threadIdx.x; b < nbuckets; b += blockDim.x) gbase[b] = off[(int64_t)b * ntiles + blockIdx.x];
   __syncwarp();
-  const int64_t cbase = (int64_t)blockIdx.x * kPartTile + (int64_t)w * kPartWarpChunk;
+  const int64_t tbase = (int64_t)blockIdx.x * kPartTile;
+  const int64_t cbase = tbase + (int64_t)w * kPartWarpChunk;
+  const uint32_t lt = lanemask_lt();
   uint32_t rank[kPartItems];
   uint32_t bk[kPartItems];
+  uint64_t va[kPartItems], vb[kPartItems];
 #pragma unroll
   for (int r = 0; r < kPartItems; r++) {
     int64_t k = cbase + r * 32 + lane;
     bool valid = k < n;
-    uint32_t b = valid ? bucket(k) : 0xFFFFFFFFu;
+    uint32_t b = 0;
+    if (valid) {
+      b = bucket(k);
+      move.load(k, va[r], vb[r]);
+    }
     // lanes with the same bucket: one ballot per bucket bit (match.any is
     // slow when a warp holds many distinct values); invalid lanes use 256
     uint32_t peers = kFull;
@@ -255,32 +273,50 @@ __global__ void __launch_bounds__(kPartThreads) k_part_scatter(BucketF bucket, M
         peers &= x ? bb : ~bb;
       }
     }
-    uint32_t before = wrun[w][valid ? b : 0];
+    uint32_t before = wrun[w * 256 + b];
     __syncwarp();
     if (valid) {
-      rank[r] = before + __popc(peers & lanemask_lt());
+      rank[r] = before + __popc(peers & lt);
       // the highest peer lane publishes the new running count
-      if ((peers >> lane) == 1u) wrun[w][b] = before + __popc(peers);
+      if ((peers >> lane) == 1u) wrun[w * 256 + b] = before + __popc(peers);
     }
-    bk[r] = b;
+    bk[r] = valid ? b : 0xFFFFFFFFu;
     __syncwarp();
   }
   __syncthreads();
-  // exclusive scan over warps per bucket (thread b handles bucket b)
-  for (int b = threadIdx.x; b < nbuckets; b += blockDim.x) {
-    uint32_t s = base_s[b];
-#pragma unroll
-    for (int ww = 0; ww < kPartWarps; ww++) {
-      uint32_t c = wrun[ww][b];
-      wrun[ww][b] = s;
-      s += c;
+  // tile-local bucket starts and per-warp offsets (thread b: bucket b)
+  {
+    const int b = threadIdx.x;  // kPartThreads == 256 buckets max
+    uint32_t tot = 0;
+    if (b < nbuckets)
+      for (int ww = 0; ww < kPartWarps; ww++) tot += wrun[ww * 256 + b];
+    uint32_t all;
+    const uint32_t ls = block_excl_scan<uint32_t>(tot, scan_sm, &all);
+    if (b < nbuckets) {
+      lstart[b] = ls;
+      uint32_t sacc = ls;
+      for (int ww = 0; ww < kPartWarps; ww++) {
+        const uint32_t c = wrun[ww * 256 + b];
+        wrun[ww * 256 + b] = sacc;
+        sacc += c;
+      }
     }
   }
   __syncthreads();
 #pragma unroll
   for (int r = 0; r < kPartItems; r++) {
-    int64_t k = cbase + r * 32 + lane;
-    if (k < n) move(k, (int64_t)wrun[w][bk[r]] + rank[r]);
+    if (bk[r] != 0xFFFFFFFFu) {
+      const uint32_t lp = wrun[w * 256 + bk[r]] + rank[r];
+      sa[lp] = va[r];
+      sb[lp] = vb[r];
+      sbk[lp] = (uint16_t)bk[r];
+    }
+  }
+  __syncthreads();
+  const int64_t tn = n - tbase < kPartTile ? n - tbase : kPartTile;
+  for (int t = threadIdx.x; t < tn; t += kPartThreads) {
+    const uint32_t b = sbk[t];
+    move.store((int64_t)gbase[b] + (t - lstart[b]), sa[t], sb[t]);
   }
 }
 
@@ -306,7 +342,10 @@ cudaError_t partition_stable(BucketF bucket, MoveF move, int64_t n, int nbuckets
   uint32_t* sc = hist + m + 1;
   cudaError_t err = scan_apply<uint32_t>(ReadU32{hist}, m, sc, WriteU32{hist}, st);
   if (err != cudaSuccess) return err;
-  k_part_scatter<BucketF, MoveF><<<(unsigned)nt, kPartThreads, 0, st>>>(bucket, move, n, nbuckets, nt, hist);
+  err = cudaFuncSetAttribute(k_part_scatter<BucketF, MoveF>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)kPartSmem);
+  if (err != cudaSuccess) return err;
+  k_part_scatter<BucketF, MoveF><<<(unsigned)nt, kPartThreads, kPartSmem, st>>>(bucket, move, n, nbuckets, nt, hist);
   return cudaGetLastError();
 }
 
