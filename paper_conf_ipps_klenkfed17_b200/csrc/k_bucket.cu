@@ -28,11 +28,15 @@
 
 namespace mm {
 
-// bucket hash: decorrelated from mm_route's owner hash (top bits of
-// header_hash), so the shard a rank owns still spreads over all buckets
+// Bucket hash: Fibonacci (multiply-shift) hashing of the 64-bit tuple -- a
+// handful of instructions instead of three Jenkins rounds, and independent of
+// mm_route's owner hash (Jenkins), so the shard a rank owns still spreads over
+// all buckets.  It is computed once per element (first partition pass) and
+// then carried in the payload's high half.
 __device__ __forceinline__ uint32_t bucket_of(uint64_t h, int nb) {
-  return jenkins32(header_hash(h) ^ 0x5bd1e995u) >> (32 - nb);
+  return (uint32_t)((h * 0x9E3779B97F4A7C15ull) >> (64 - nb));
 }
+
 
 struct SnapRead {
   Side S;
@@ -40,39 +44,46 @@ struct SnapRead {
   __device__ __forceinline__ uint64_t hdr(int64_t u) const { return S.hdr(0, u, resid, pb); }
 };
 
+// payload of a partitioned element: header word + (bucket << 32 | snapshot index)
 template <bool FIRST>
 struct BDigit {
   SnapRead snap;
-  const uint64_t* h;
+  const uint64_t* bi;
   int nb, shift, dmask;
   __device__ __forceinline__ uint32_t operator()(int64_t k) const {
-    const uint64_t x = FIRST ? snap.hdr(k) : h[k];
-    return (bucket_of(x, nb) >> shift) & (uint32_t)dmask;
+    const uint32_t b = FIRST ? bucket_of(snap.hdr(k), nb) : (uint32_t)(bi[k] >> 32);
+    return (b >> shift) & (uint32_t)dmask;
   }
 };
 template <bool FIRST>
 struct BMove {
   SnapRead snap;
   const uint64_t* h;
-  const uint32_t* ix;
+  const uint64_t* bi;
+  int nb;
   uint64_t* oh;
-  uint32_t* oi;
+  uint64_t* obi;
   __device__ __forceinline__ void load(int64_t k, uint64_t& a, uint64_t& b) const {
-    a = FIRST ? snap.hdr(k) : h[k];
-    b = FIRST ? (uint64_t)k : ix[k];
+    if (FIRST) {
+      a = snap.hdr(k);
+      b = ((uint64_t)bucket_of(a, nb) << 32) | (uint64_t)k;
+    } else {
+      a = h[k];
+      b = bi[k];
+    }
   }
   __device__ __forceinline__ void store(int64_t dst, uint64_t a, uint64_t b) const {
     oh[dst] = a;
-    oi[dst] = (uint32_t)b;
+    obi[dst] = b;
   }
 };
 
 // off[b] = first position of bucket b in the bucket-sorted array (b in 0..B).
-__global__ void k_bucket_bounds(const uint64_t* h, int64_t n, int nb, uint32_t* off) {
+__global__ void k_bucket_bounds(const uint64_t* bi, int64_t n, int nb, uint32_t* off) {
   const uint32_t B = 1u << nb;
   for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < n; p += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t b = bucket_of(h[p], nb);
-    const uint32_t prev = p == 0 ? 0xFFFFFFFFu : bucket_of(h[p - 1], nb);
+    const uint32_t b = (uint32_t)(bi[p] >> 32);
+    const uint32_t prev = p == 0 ? 0xFFFFFFFFu : (uint32_t)(bi[p - 1] >> 32);
     if (b != prev)
       for (uint32_t x = prev + 1; x <= b; x++) off[x] = (uint32_t)p;  // (prev+1 wraps to 0 at p == 0)
     if (p == n - 1)
@@ -90,8 +101,8 @@ static int grid_cap(int64_t n, int threads) {
 }
 
 // Partition one side of the snapshot into bucket order.
-static cudaError_t partition_side(const SnapRead& snap, int64_t n, int nb, uint64_t* h0, uint32_t* i0, uint64_t* h1,
-                                  uint32_t* i1, uint32_t* part, uint32_t* off, uint64_t** out_h, uint32_t** out_i,
+static cudaError_t partition_side(const SnapRead& snap, int64_t n, int nb, uint64_t* h0, uint64_t* i0, uint64_t* h1,
+                                  uint64_t* i1, uint32_t* part, uint32_t* off, uint64_t** out_h, uint64_t** out_i,
                                   cudaStream_t st) {
   const uint32_t B = 1u << nb;
   if (n == 0) {
@@ -104,7 +115,7 @@ static cudaError_t partition_side(const SnapRead& snap, int64_t n, int nb, uint6
   const int passes = (nb + 7) / 8;
   const int dbits = (nb + passes - 1) / passes;
   uint64_t* hb[2] = {h0, h1};
-  uint32_t* ib[2] = {i0, i1};
+  uint64_t* ib[2] = {i0, i1};
   int cur = 0;
   cudaError_t err;
   for (int p = 0; p < passes; p++) {
@@ -113,16 +124,16 @@ static cudaError_t partition_side(const SnapRead& snap, int64_t n, int nb, uint6
     const int nbk = 1 << bits;
     if (p == 0) {
       err = partition_stable(BDigit<true>{snap, nullptr, nb, shift, nbk - 1},
-                             BMove<true>{snap, nullptr, nullptr, hb[cur], ib[cur]}, n, nbk, part, st);
+                             BMove<true>{snap, nullptr, nullptr, nb, hb[cur], ib[cur]}, n, nbk, part, st);
     } else {
-      err = partition_stable(BDigit<false>{snap, hb[cur], nb, shift, nbk - 1},
-                             BMove<false>{snap, hb[cur], ib[cur], hb[cur ^ 1], ib[cur ^ 1]}, n, nbk, part, st);
+      err = partition_stable(BDigit<false>{snap, ib[cur], nb, shift, nbk - 1},
+                             BMove<false>{snap, hb[cur], ib[cur], nb, hb[cur ^ 1], ib[cur ^ 1]}, n, nbk, part, st);
       cur ^= 1;
     }
     if (err != cudaSuccess) return err;
   }
   count_launch();
-  k_bucket_bounds<<<grid_cap(n, 256), 256, 0, st>>>(hb[cur], n, nb, off);
+  k_bucket_bounds<<<grid_cap(n, 256), 256, 0, st>>>(ib[cur], n, nb, off);
   *out_h = hb[cur];
   *out_i = ib[cur];
   return cudaGetLastError();
@@ -136,10 +147,10 @@ constexpr uint32_t kBucketH = 4096;  // hash slots (>= 2 * kBucketCap)
 struct BucketArgs {
   FlatArgs a;
   const uint64_t* rh;  // bucket-sorted receive headers
-  const uint32_t* ri;  // their snapshot indices
+  const uint64_t* ri;  // (bucket << 32) | snapshot index
   const uint32_t* roff;
   const uint64_t* mh;
-  const uint32_t* mi;
+  const uint64_t* mi;
   const uint32_t* moff;
   uint32_t* overflow;
 };
@@ -186,10 +197,10 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
   for (uint32_t e = tid; e < n; e += NT) {
     if (e < nr) {
       sm.hdr[e] = ba.rh[r0 + e];
-      sm.idx[e] = ba.ri[r0 + e];
+      sm.idx[e] = (uint32_t)ba.ri[r0 + e];
     } else {
       sm.hdr[e] = ba.mh[m0 + e - nr];
-      sm.idx[e] = ba.mi[m0 + e - nr];
+      sm.idx[e] = (uint32_t)ba.mi[m0 + e - nr];
     }
   }
   for (uint32_t s = tid; s < kBucketH / 2; s += NT) reinterpret_cast<uint32_t*>(sm.table)[s] = 0xFFFFFFFFu;
@@ -198,7 +209,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
   // message tuples into the hash table
   for (uint32_t e = nr + tid; e < n; e += NT) {
     const uint64_t h = sm.hdr[e];
-    uint32_t s = header_hash(h) & hmask;
+    uint32_t s = slot_hash(h) & hmask;
     while (true) {
       uint16_t o = sm.table[s];
       if (o == kEmpty16) {
@@ -237,7 +248,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
       k = sm.slot_id[sm.key[e]];
     } else {
       const uint64_t h = sm.hdr[e];
-      uint32_t s = header_hash(h) & hmask;
+      uint32_t s = slot_hash(h) & hmask;
       k = kNone;
       while (true) {
         const uint16_t o = sm.table[s];
@@ -351,7 +362,7 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cuda
   rs.pb = 0;  // single endpoint: pending batch starts at 0
   ms.pb = 0;
   uint64_t *rh, *mh;
-  uint32_t *ri, *mi;
+  uint64_t *ri, *mi;
   cudaError_t err = partition_side(rs, a.nr, nb, s.h[0], s.i[0], s.h[1], s.i[1], s.part, s.roff, &rh, &ri, st);
   if (err != cudaSuccess) return err;
   err = partition_side(ms, a.nm, nb, s.h[2], s.i[2], s.h[3], s.i[3], s.part, s.moff, &mh, &mi, st);
@@ -388,7 +399,7 @@ struct SortedCompactOut {
   Side S;
   int64_t resid;
   const uint64_t* h;
-  const uint32_t* ix;
+  const uint64_t* ix;
   int64_t n;
   uint64_t* q_h;
   int64_t* q_c;
@@ -396,14 +407,14 @@ struct SortedCompactOut {
   __device__ __forceinline__ void operator()(int64_t p, uint32_t ex, uint32_t v) const {
     if (v) {
       q_h[ex] = h[p];
-      q_c[ex] = S.cookie(0, ix[p], resid, 0);
+      q_c[ex] = S.cookie(0, (uint32_t)ix[p], resid, 0);
     }
     if (p == n - 1) *q_len = (int32_t)(ex + v);
   }
 };
 __global__ void k_set_len0(int32_t* q_len) { *q_len = 0; }
 
-cudaError_t run_compact_sorted(const Side& S, int64_t resid, int64_t n, const uint64_t* h, const uint32_t* ix,
+cudaError_t run_compact_sorted(const Side& S, int64_t resid, int64_t n, const uint64_t* h, const uint64_t* ix,
                                const uint8_t* matched, uint64_t* q_h, int64_t* q_c, int32_t* q_len, uint32_t* scan,
                                cudaStream_t st) {
   if (n == 0) {

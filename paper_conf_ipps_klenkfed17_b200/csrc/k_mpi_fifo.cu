@@ -270,7 +270,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     // P2 -------------------------------------------------------------------
     for (int64_t j = tid; j < nm; j += NT) {
       const uint64_t h = ws.msgs[j];
-      uint32_t s = header_hash(h) & hmask;
+      uint32_t s = slot_hash(h) & hmask;
       while (true) {
         uint16_t o = ws.table[s];
         if (o == kEmpty16) {
@@ -322,7 +322,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         rk = kWild;
       } else {
         rk = kNone;
-        uint32_t s = header_hash(h) & hmask;
+        uint32_t s = slot_hash(h) & hmask;
         while (true) {
           const uint16_t o = ws.table[s];
           if (o == kEmpty16) break;
@@ -432,7 +432,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         __syncthreads();
         for (uint32_t k = tid; k < K; k += NT) {
           const uint64_t gk = ws.keyhdr[k] & gmsk;
-          uint32_t sl = header_hash(gk) & hmask;
+          uint32_t sl = slot_hash(gk) & hmask;
           while (true) {
             uint16_t o = ws.table[sl];
             if (o == kEmpty16) {
@@ -470,7 +470,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         }
         for (uint32_t x = tid; x < W; x += NT) {
           const uint64_t rg = ws.recvs[ws.wl[x]] & gmsk;
-          uint32_t sl = header_hash(rg) & hmask;
+          uint32_t sl = slot_hash(rg) & hmask;
           uint16_t g = kNone;
           while (true) {
             const uint16_t o = ws.table[sl];

@@ -282,7 +282,7 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
          ensure(e->scan, (size_t)scan_scratch_elems(n) * 8) == cudaSuccess;
     for (int b = 0; ok && b < 4; b++) {
       const int64_t c = b < 2 ? e->rcap : e->mcap;
-      ok = ensure(e->bh[b], c * 8) == cudaSuccess && ensure(e->bi[b], c * 4) == cudaSuccess;
+      ok = ensure(e->bh[b], c * 8) == cudaSuccess && ensure(e->bi[b], c * 8) == cudaSuccess;
     }
     ok = ok && ensure(e->bpart, (size_t)partition_scratch_elems(e->rcap > e->mcap ? e->rcap : e->mcap) * 4) == cudaSuccess &&
          ensure(e->broff, (size_t)bucket_scratch_elems(n) * 4) == cudaSuccess &&
@@ -505,7 +505,7 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
   if (e->flat_kernel == MM_FLAT_KERNEL_BUCKETED) {
     for (int b = 0; b < 4; b++) {
       bs.h[b] = (uint64_t*)e->bh[b].p;
-      bs.i[b] = (uint32_t*)e->bi[b].p;
+      bs.i[b] = (uint64_t*)e->bi[b].p;
     }
     bs.part = (uint32_t*)e->bpart.p;
     bs.roff = (uint32_t*)e->broff.p;

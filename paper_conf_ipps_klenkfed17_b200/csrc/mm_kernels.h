@@ -94,7 +94,7 @@ cudaError_t run_hash(const FlatArgs& a, const HashScratch& h, cudaStream_t st);
 // not fit on chip (the caller then falls back to run_sort_rank / run_hash).
 struct BucketScratch {
   uint64_t* h[4];  // receive ping-pong (0,1), message ping-pong (2,3)
-  uint32_t* i[4];
+  uint64_t* i[4];  // (bucket << 32) | snapshot index
   uint32_t* part;
   uint32_t* roff;
   uint32_t* moff;
@@ -102,12 +102,12 @@ struct BucketScratch {
   int64_t rres, mres;
   // outputs: the bucket-sorted sides (results are written in this order)
   const uint64_t* rh_sorted;
-  const uint32_t* ri_sorted;
+  const uint64_t* ri_sorted;
   const uint64_t* mh_sorted;
-  const uint32_t* mi_sorted;
+  const uint64_t* mi_sorted;
 };
 cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cudaStream_t st);
-cudaError_t run_compact_sorted(const Side& S, int64_t resid, int64_t n, const uint64_t* h, const uint32_t* ix,
+cudaError_t run_compact_sorted(const Side& S, int64_t resid, int64_t n, const uint64_t* h, const uint64_t* ix,
                                const uint8_t* matched, uint64_t* q_h, int64_t* q_c, int32_t* q_len, uint32_t* scan,
                                cudaStream_t st);
 int64_t bucket_scratch_elems(int64_t n);

@@ -11,6 +11,12 @@ constexpr uint16_t kWild = 0xFFFEu;
 constexpr uint16_t kNone = 0xFFFFu;
 constexpr uint16_t kEmpty16 = 0xFFFFu;
 
+// Slot of a tuple in an on-chip hash table: multiply-shift of the 64-bit word
+// (a few instructions; the tables are small and private to one CTA).
+__device__ __forceinline__ uint32_t slot_hash(uint64_t h) {
+  return (uint32_t)((h * 0xD6E8FEB86659FD93ull) >> 40);
+}
+
 // 16-bit CAS through the containing 32-bit word.
 // (pointer arithmetic, not integer casts, so shared-memory provenance survives
 // and the atomics compile to ATOMS)
