@@ -41,14 +41,17 @@ def launches(path, out):
     hi = [i for i, r in enumerate(rows) if "Kernel Name" in r][0]
     h = rows[hi]
     ki, vi, ui = h.index("Kernel Name"), h.index("Metric Value"), h.index("Metric Unit")
+    mi = h.index("Metric Name") if "Metric Name" in h else None
     agg = collections.OrderedDict()
     for r in rows[hi + 1:]:
         if len(r) <= vi:
             continue
+        if mi is not None and r[mi] != "gpu__time_duration.sum":
+            continue
         name = r[ki].split("(")[0]
         v = float(r[vi].replace(",", ""))
         unit = r[ui]
-        v = v / 1e3 if unit == "nsecond" else v * (1e3 if unit == "msecond" else 1.0)  # -> us
+        v = v * {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3}.get(unit, 1e-3)
         a = agg.setdefault(name, [0, 0.0])
         a[0] += 1
         a[1] += v
