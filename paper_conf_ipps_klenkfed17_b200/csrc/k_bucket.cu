@@ -112,7 +112,7 @@ static cudaError_t partition_side(const SnapRead& snap, int64_t n, int nb, uint6
     *out_i = i0;
     return cudaGetLastError();
   }
-  const int passes = (nb + 7) / 8;
+  const int passes = (nb + 8) / 9;  // up to 9 bits (512 buckets) per pass
   const int dbits = (nb + passes - 1) / passes;
   uint64_t* hb[2] = {h0, h1};
   uint64_t* ib[2] = {i0, i1};
@@ -140,9 +140,9 @@ static cudaError_t partition_side(const SnapRead& snap, int64_t n, int nb, uint6
 }
 
 // ------------------------------------------------------------- bucket kernel
-constexpr int kBucketCap = 2048;   // elements (receives + messages) per bucket on chip
+constexpr int kBucketCap = 1024;   // elements (receives + messages) per bucket on chip
 constexpr int kBucketThreads = 256;
-constexpr uint32_t kBucketH = 4096;  // hash slots (>= 2 * kBucketCap)
+constexpr uint32_t kBucketH = 2048;  // hash slots (>= 2 * kBucketCap)
 
 struct BucketArgs {
   FlatArgs a;
@@ -347,9 +347,11 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
   if (lane == 0 && nmatch) atomicAdd(a.n_matched, (unsigned long long)nmatch);
 }
 
+// ~512 elements per bucket on average (capacity 1024: a bucket overflows
+// only for heavily repeated tuples)
 int64_t bucket_bits_for(int64_t n) {
   int nb = 1;
-  while (nb < 24 && ((int64_t)1 << nb) * 1024 < n) nb++;
+  while (nb < 27 && ((int64_t)1 << nb) * 512 < n) nb++;
   return nb;
 }
 

@@ -195,14 +195,15 @@ cudaError_t scan_apply(In in, int64_t n, T* scratch /* >= ntiles + 1 */, Out out
 inline int64_t scan_scratch_elems(int64_t n) { return (n + kScanTile - 1) / kScanTile + 2; }
 
 // ---------------------------------------------- stable bucket partition
-// Stable counting-sort scatter of n elements into up to 256 buckets.  Used by
+// Stable counting-sort scatter of n elements into up to 512 buckets.  Used by
 // the LSD radix passes of the ordered no-wildcard level (row A4) and by
 // mm_route (row A6).  Tile = 8 warps x 512 contiguous elements; each warp owns
 // a contiguous chunk and keeps private running counts per bucket, so ranks are
 // stable without CTA-wide barriers inside the tile.
 constexpr int kPartWarps = 8;
 constexpr int kPartThreads = kPartWarps * 32;
-constexpr int kPartItems = 16;                          // per lane
+constexpr int kPartItems = 8;                           // per lane
+constexpr int kPartMaxBuckets = 512;
 constexpr int kPartWarpChunk = 32 * kPartItems;         // 512
 constexpr int kPartTile = kPartWarps * kPartWarpChunk;  // 4096
 
@@ -210,8 +211,8 @@ constexpr int kPartTile = kPartWarps * kPartWarpChunk;  // 4096
 template <class BucketF>
 __global__ void __launch_bounds__(kPartThreads) k_part_hist(BucketF bucket, int64_t n, int nbuckets, int64_t ntiles,
                                                             uint32_t* hist) {
-  __shared__ uint32_t h[256];
-  for (int b = threadIdx.x; b < 256; b += blockDim.x) h[b] = 0;
+  __shared__ uint32_t h[kPartMaxBuckets];
+  for (int b = threadIdx.x; b < kPartMaxBuckets; b += blockDim.x) h[b] = 0;
   __syncthreads();
   const int64_t base = (int64_t)blockIdx.x * kPartTile;
 #pragma unroll 4
@@ -229,7 +230,7 @@ __global__ void __launch_bounds__(kPartThreads) k_part_hist(BucketF bucket, int6
 // then written out so that consecutive threads write consecutive addresses of
 // a bucket's run (coalesced stores instead of one scattered store per lane).
 // move.load(k, a, b) reads element k's payload, move.store(dst, a, b) writes it.
-constexpr size_t kPartSmem = (size_t)kPartTile * (8 + 8 + 2) + (kPartWarps + 3) * 256 * 4 + 64;
+constexpr size_t kPartSmem = (size_t)kPartTile * (8 + 8 + 2) + (kPartWarps + 2) * kPartMaxBuckets * 4 + 64 * 4 + 16;
 
 template <class BucketF, class MoveF>
 __global__ void __launch_bounds__(kPartThreads) k_part_scatter(BucketF bucket, MoveF move, int64_t n, int nbuckets,
@@ -237,13 +238,13 @@ __global__ void __launch_bounds__(kPartThreads) k_part_scatter(BucketF bucket, M
   extern __shared__ __align__(16) uint8_t part_smem[];
   uint64_t* sa = reinterpret_cast<uint64_t*>(part_smem);
   uint64_t* sb = sa + kPartTile;
-  uint32_t* wrun = reinterpret_cast<uint32_t*>(sb + kPartTile);  // [kPartWarps][256]
-  uint32_t* lstart = wrun + kPartWarps * 256;                     // tile-local bucket starts
-  uint32_t* gbase = lstart + 256;                                 // global bucket bases
-  uint32_t* scan_sm = gbase + 256;
+  uint32_t* wrun = reinterpret_cast<uint32_t*>(sb + kPartTile);  // [kPartWarps][kPartMaxBuckets]
+  uint32_t* lstart = wrun + kPartWarps * kPartMaxBuckets;         // tile-local bucket starts
+  uint32_t* gbase = lstart + kPartMaxBuckets;                     // global bucket bases
+  uint32_t* scan_sm = gbase + kPartMaxBuckets;
   uint16_t* sbk = reinterpret_cast<uint16_t*>(scan_sm + 64);
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  for (int b = lane; b < 256; b += 32) wrun[w * 256 + b] = 0;
+  for (int b = lane; b < kPartMaxBuckets; b += 32) wrun[w * kPartMaxBuckets + b] = 0;
   for (int b = threadIdx.x; b < nbuckets; b += blockDim.x) gbase[b] = off[(int64_t)b * ntiles + blockIdx.x];
   __syncwarp();
   const int64_t tbase = (int64_t)blockIdx.x * kPartTile;
@@ -262,51 +263,63 @@ __global__ void __launch_bounds__(kPartThreads) k_part_scatter(BucketF bucket, M
       move.load(k, va[r], vb[r]);
     }
     // lanes with the same bucket: one ballot per bucket bit (match.any is
-    // slow when a warp holds many distinct values); invalid lanes use 256
+    // slow when a warp holds many distinct values); invalid lanes use 512
     uint32_t peers = kFull;
     {
-      const uint32_t v = valid ? b : 256u;
+      const uint32_t v = valid ? b : (uint32_t)kPartMaxBuckets;
 #pragma unroll
-      for (int bit = 0; bit < 9; bit++) {
+      for (int bit = 0; bit < 10; bit++) {
         const bool x = (v >> bit) & 1u;
         const uint32_t bb = __ballot_sync(kFull, x);
         peers &= x ? bb : ~bb;
       }
     }
-    uint32_t before = wrun[w * 256 + b];
+    uint32_t before = wrun[w * kPartMaxBuckets + b];
     __syncwarp();
     if (valid) {
       rank[r] = before + __popc(peers & lt);
       // the highest peer lane publishes the new running count
-      if ((peers >> lane) == 1u) wrun[w * 256 + b] = before + __popc(peers);
+      if ((peers >> lane) == 1u) wrun[w * kPartMaxBuckets + b] = before + __popc(peers);
     }
     bk[r] = valid ? b : 0xFFFFFFFFu;
     __syncwarp();
   }
   __syncthreads();
-  // tile-local bucket starts and per-warp offsets (thread b: bucket b)
+  // tile-local bucket starts and per-warp offsets (thread t: buckets 2t, 2t+1)
   {
-    const int b = threadIdx.x;  // kPartThreads == 256 buckets max
-    uint32_t tot = 0;
-    if (b < nbuckets)
-      for (int ww = 0; ww < kPartWarps; ww++) tot += wrun[ww * 256 + b];
+    constexpr int BPT = kPartMaxBuckets / kPartThreads;
+    uint32_t tot[BPT];
+    uint32_t sum = 0;
+#pragma unroll
+    for (int j = 0; j < BPT; j++) {
+      const int b = threadIdx.x * BPT + j;
+      tot[j] = 0;
+      if (b < nbuckets)
+        for (int ww = 0; ww < kPartWarps; ww++) tot[j] += wrun[ww * kPartMaxBuckets + b];
+      sum += tot[j];
+    }
     uint32_t all;
-    const uint32_t ls = block_excl_scan<uint32_t>(tot, scan_sm, &all);
-    if (b < nbuckets) {
-      lstart[b] = ls;
-      uint32_t sacc = ls;
-      for (int ww = 0; ww < kPartWarps; ww++) {
-        const uint32_t c = wrun[ww * 256 + b];
-        wrun[ww * 256 + b] = sacc;
-        sacc += c;
+    uint32_t ls = block_excl_scan<uint32_t>(sum, scan_sm, &all);
+#pragma unroll
+    for (int j = 0; j < BPT; j++) {
+      const int b = threadIdx.x * BPT + j;
+      if (b < nbuckets) {
+        lstart[b] = ls;
+        uint32_t sacc = ls;
+        for (int ww = 0; ww < kPartWarps; ww++) {
+          const uint32_t c = wrun[ww * kPartMaxBuckets + b];
+          wrun[ww * kPartMaxBuckets + b] = sacc;
+          sacc += c;
+        }
       }
+      ls += tot[j];
     }
   }
   __syncthreads();
 #pragma unroll
   for (int r = 0; r < kPartItems; r++) {
     if (bk[r] != 0xFFFFFFFFu) {
-      const uint32_t lp = wrun[w * 256 + bk[r]] + rank[r];
+      const uint32_t lp = wrun[w * kPartMaxBuckets + bk[r]] + rank[r];
       sa[lp] = va[r];
       sb[lp] = vb[r];
       sbk[lp] = (uint16_t)bk[r];
@@ -330,7 +343,7 @@ struct WriteU32 {
 };
 
 template <class BucketF, class MoveF>
-cudaError_t partition_stable(BucketF bucket, MoveF move, int64_t n, int nbuckets, uint32_t* hist /* 256*ntiles+2 */,
+cudaError_t partition_stable(BucketF bucket, MoveF move, int64_t n, int nbuckets, uint32_t* hist /* see partition_scratch_elems */,
                              cudaStream_t st) {
   if (n <= 0) return cudaSuccess;
   int64_t nt = (n + kPartTile - 1) / kPartTile;
@@ -351,7 +364,7 @@ cudaError_t partition_stable(BucketF bucket, MoveF move, int64_t n, int nbuckets
 
 inline int64_t partition_scratch_elems(int64_t n) {
   int64_t nt = (n + kPartTile - 1) / kPartTile;
-  int64_t m = 256 * nt;
+  int64_t m = kPartMaxBuckets * nt;
   return m + 1 + scan_scratch_elems(m);
 }
 
