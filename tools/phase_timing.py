@@ -22,9 +22,10 @@ for it in range(3):
     eng.reset(); eng.post_recvs(rh, None, ro); eng.push_msgs(mh, None, mo); eng.match_batch(orc, omc)
     torch.cuda.synchronize()
     L.mm_debug_phase_cycles(buf.ctypes.data, 1)
-tot = buf[:11].sum()
+tot = buf[:12].sum()
 names = ["prologue", "P1 stage", "P2 insert", "P3 ids", "P4 classify", "P5 scans", "P6 place", "P7 wildcards",
-         "P8 resolve+out", "P9 msg compact", "P7a group setup"]
+         "P8 resolve+out", "P9 msg compact", "P7a group setup", "P7 K<=32 chain"]
 for i, nm in enumerate(names):
     print("%-16s %8.0f cycles/endpoint  %5.1f%%" % (nm, buf[i] / q.n_endpoints, 100.0 * buf[i] / tot))
 print("total %.0f cycles per endpoint (per CTA, thread 0)" % (tot / q.n_endpoints))
+print("endpoints on the K<=32 chain: %d, on the group path: %d" % (buf[13], buf[14]))
