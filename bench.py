@@ -44,6 +44,11 @@ WORKLOADS = {
 }
 
 
+def coll_device():
+    import torch.distributed as dist
+    return "cuda" if dist.get_backend() == "nccl" else "cpu"
+
+
 def dist_env():
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -269,7 +274,7 @@ def timed(args, step, eng, world, query=True):
         dist.barrier()
     t = e0.elapsed_time(e1)
     if world > 1:
-        tt = torch.tensor([t], dtype=torch.float64, device="cuda")
+        tt = torch.tensor([t], dtype=torch.float64, device=coll_device())
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         t = float(tt.item())
     out = {"t_ms": t}
@@ -287,7 +292,7 @@ def finish_level(res, world, peak, level):
     matches = res["matches_per_step"]
     total = matches
     if world > 1:
-        t = torch.tensor([matches], dtype=torch.int64, device="cuda")
+        t = torch.tensor([matches], dtype=torch.int64, device=coll_device())
         dist.all_reduce(t)
         total = int(t.item())
     steps = res["steps"] if "steps" in res else None
@@ -383,10 +388,15 @@ def main():
         run_reference(args, world, rank)
         return
     import torch
-    torch.cuda.set_device(local)
+    torch.cuda.set_device(local % max(1, torch.cuda.device_count()))
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        # MM_BENCH_BACKEND=gloo: several ranks sharing one GPU (path testing only)
+        backend = os.environ.get("MM_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     peak = load_peaks()
     clocks = Clocks(local)
     clocks.start()

@@ -68,18 +68,29 @@ class ShardedMatcher:
         self._mseq = 0
 
     def _exchange(self, tensors, counts):
-        """all-to-all of equally split tensors; counts[d] elements go to rank d."""
+        """all-to-all of equally split tensors; counts[d] elements go to rank d.
+        With NCCL the device tensors are exchanged directly over NVLink; with
+        gloo (CPU testing, or several ranks sharing one GPU) they are staged
+        through host memory."""
+        host = dist.get_backend(self.group) == "gloo"
         send = counts.to(torch.int64)
+        if host:
+            send = send.cpu()
         recv = torch.empty_like(send)
         dist.all_to_all_single(recv, send, group=self.group)
-        splits = torch.stack([send, recv]).cpu()  # one host round trip for both
+        splits = torch.stack([send.cpu(), recv.cpu()])  # one host round trip for both
         in_splits = splits[0].tolist()
         out_splits = splits[1].tolist()
         n_out = int(sum(out_splits))
         outs = []
         for t in tensors:
             o = self.ops.empty(n_out, t)
-            dist.all_to_all_single(o, t, out_splits, in_splits, group=self.group)
+            if host and t.is_cuda:
+                oc = torch.empty(n_out, dtype=t.dtype)
+                dist.all_to_all_single(oc, t.cpu(), out_splits, in_splits, group=self.group)
+                o.copy_(oc)
+            else:
+                dist.all_to_all_single(o, t, out_splits, in_splits, group=self.group)
             outs.append(o)
         return outs
 
