@@ -204,9 +204,12 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
     }
   }
   for (uint32_t s = tid; s < kBucketH / 2; s += NT) reinterpret_cast<uint32_t*>(sm.table)[s] = 0xFFFFFFFFu;
-  if (tid == 0) sm.matched = 0;
+  if (tid == 0) {
+    sm.matched = 0;
+    sm.K = 0;
+  }
   __syncthreads();
-  // message tuples into the hash table
+  // message tuples into the hash table; the CAS winner takes the next dense id
   for (uint32_t e = nr + tid; e < n; e += NT) {
     const uint64_t h = sm.hdr[e];
     uint32_t s = slot_hash(h) & hmask;
@@ -214,29 +217,18 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
       uint16_t o = sm.table[s];
       if (o == kEmpty16) {
         o = cas16(&sm.table[s], kEmpty16, (uint16_t)e);
-        if (o == kEmpty16) break;
+        if (o == kEmpty16) {
+          const uint32_t id = atomicAdd(&sm.K, 1u);
+          sm.slot_id[s] = (uint16_t)id;
+#pragma unroll
+          for (int q = 0; q < (ORDERED ? 8 : 2); q++) sm.pcnt[q][id] = 0;
+          break;
+        }
       }
       if (sm.hdr[o] == h) break;
       s = (s + 1) & hmask;
     }
     sm.key[e] = (uint16_t)s;
-  }
-  __syncthreads();
-  {  // dense tuple ids
-    constexpr uint32_t per = kBucketH / NT;
-    const uint32_t s0 = tid * per;
-    uint32_t c = 0;
-    for (uint32_t s = s0; s < s0 + per; s++) c += sm.table[s] != kEmpty16;
-    uint32_t tot;
-    uint32_t id = block_excl_scan<uint32_t>(c, sm.scan, &tot);
-    for (uint32_t s = s0; s < s0 + per; s++)
-      if (sm.table[s] != kEmpty16) {
-        sm.slot_id[s] = (uint16_t)id;
-#pragma unroll
-        for (int q = 0; q < (ORDERED ? 8 : 2); q++) sm.pcnt[q][id] = 0;
-        id++;
-      }
-    if (tid == 0) sm.K = tot;
   }
   __syncthreads();
   const uint32_t K = sm.K;

@@ -284,10 +284,15 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     stage_side<NT>(a.R, e, nr, rres, rpb, ws.recvs, tid);
     for (uint32_t s = tid; s < H / 2; s += NT) reinterpret_cast<uint32_t*>(ws.table)[s] = 0xFFFFFFFFu;
     for (int64_t k = tid; k < (nm + 31) / 32; k += NT) ws.matched[k] = 0u;
-    if (tid == 0) sh_matched = 0;
+    if (tid == 0) {
+      sh_matched = 0;
+      sh_K = 0;
+    }
     __syncthreads();
     MM_PHASE(1);
     // P2 -------------------------------------------------------------------
+    // insert message tuples; the CAS winner of a slot takes the next dense
+    // tuple id and initialises the tuple's entries (no separate id pass)
     for (int64_t j = tid; j < nm; j += NT) {
       const uint64_t h = ws.msgs[j];
       uint32_t s = slot_hash(h) & hmask;
@@ -295,7 +300,16 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         uint16_t o = ws.table[s];
         if (o == kEmpty16) {
           o = cas16(&ws.table[s], kEmpty16, (uint16_t)j);
-          if (o == kEmpty16) break;
+          if (o == kEmpty16) {
+            const uint32_t id = atomicAdd(&sh_K, 1u);
+            ws.slot_id[s] = (uint16_t)id;
+            ws.keyhdr[id] = h;
+#pragma unroll
+            for (int q = 0; q < 8; q++) ws.pcnt[q * ws.mcap + id] = 0;
+            ws.key_c[id] = 0;
+            ws.key_cur[id] = 0;
+            break;
+          }
         }
         if (ws.msgs[o] == h) break;
         s = (s + 1) & hmask;
@@ -304,29 +318,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     }
     __syncthreads();
     MM_PHASE(2);
-    // P3 -------------------------------------------------------------------
-    {
-      const uint32_t per = (H + NT - 1) / NT;
-      const uint32_t s0 = min(H, tid * per), s1 = min(H, s0 + per);
-      uint32_t c = 0;
-      for (uint32_t s = s0; s < s1; s++) c += ws.table[s] != kEmpty16;
-      uint32_t tot;
-      uint32_t id = block_excl_scan<uint32_t>(c, scan_sm, &tot);
-      for (uint32_t s = s0; s < s1; s++) {
-        const uint16_t o = ws.table[s];
-        if (o != kEmpty16) {
-          ws.slot_id[s] = (uint16_t)id;
-          ws.keyhdr[id] = ws.msgs[o];
-#pragma unroll
-          for (int q = 0; q < 8; q++) ws.pcnt[q * ws.mcap + id] = 0;
-          ws.key_c[id] = 0;
-          ws.key_cur[id] = 0;
-          id++;
-        }
-      }
-      if (tid == 0) sh_K = tot;
-    }
-    __syncthreads();
+    // P3 (dense ids) is folded into P2
+    MM_PHASE(3);
     const uint32_t K = sh_K;
     MM_PHASE(3);
     // P4 -------------------------------------------------------------------
