@@ -56,11 +56,9 @@ __device__ unsigned long long g_phase_cycles[16];
 
 
 struct FifoWs {
-  uint64_t* msgs;       // [mcap] staged message headers
-  uint64_t* recvs;      // [rcap] staged receive headers
+  uint64_t* whdr;       // [wcap] headers of the first wcap wildcard receives
   uint64_t* keyhdr;     // [mcap] tuple id -> header
   uint16_t* table;      // [H] slot -> representative message
-  uint16_t* slot_id;    // [H] slot -> dense tuple id
   uint16_t* key_cnt;    // [mcap] messages of tuple k
   uint16_t* key_start;  // [mcap] start of tuple k in by_key / wlog
   uint16_t* key_rcnt;   // [mcap] exact receives of tuple k
@@ -91,11 +89,9 @@ struct FifoWs {
 
 __device__ __forceinline__ FifoWs carve(uint8_t* base, const FifoLayout& L) {
   FifoWs w;
-  w.msgs = reinterpret_cast<uint64_t*>(base + L.msgs);
-  w.recvs = reinterpret_cast<uint64_t*>(base + L.recvs);
+  w.whdr = reinterpret_cast<uint64_t*>(base + L.whdr);
   w.keyhdr = reinterpret_cast<uint64_t*>(base + L.keyhdr);
   w.table = reinterpret_cast<uint16_t*>(base + L.table);
-  w.slot_id = reinterpret_cast<uint16_t*>(base + L.slot_id);
   w.key_cnt = reinterpret_cast<uint16_t*>(base + L.key_cnt);
   w.key_start = reinterpret_cast<uint16_t*>(base + L.key_start);
   w.key_rcnt = reinterpret_cast<uint16_t*>(base + L.key_rcnt);
@@ -192,9 +188,9 @@ __device__ __forceinline__ void stage_side(const Side& S, int e, int64_t n, int6
 // one redux.sync.min and a select, no shared-memory load.
 // test_admit: wildcards may differ, so each lane tests admission with the
 // masked XOR; otherwise every wildcard admits every candidate (a group).
-template <class KeyF, class PosF>
+template <class KeyF, class PosF, class HdrF>
 __device__ __forceinline__ void register_chain(const FifoWs& ws, uint32_t kn, KeyF keyof, uint32_t wn, PosF posof,
-                                               bool test_admit, int lane) {
+                                               HdrF hdrof, bool test_admit, int lane) {
   if (wn == 0) return;
   const bool own = lane < kn;
   uint32_t k = 0, cur = 0, c = 0, rs = 0, rc = 0, st = 0, cnt = 0;
@@ -213,8 +209,9 @@ __device__ __forceinline__ void register_chain(const FifoWs& ws, uint32_t kn, Ke
     if (own)
       while (cur < rc && ws.rby_key[rs + cur] < w) cur++;
   };
-  uint32_t w = posof(0);
-  uint64_t r = test_admit ? ws.recvs[w] : 0ull;
+  uint32_t x0 = posof(0);
+  uint32_t w = ws.wl[x0];
+  uint64_t r = test_admit ? hdrof(x0) : 0ull;
   advance(w);
   uint32_t h0 = head_at(cur + c), h1 = head_at(cur + c + 1), h2 = head_at(cur + c + 2);
   for (uint32_t t = 0; t < wn; t++) {
@@ -222,8 +219,9 @@ __device__ __forceinline__ void register_chain(const FifoWs& ws, uint32_t kn, Ke
     uint32_t wn1 = w, x0 = 0xFFFFFFFFu, x1 = 0xFFFFFFFFu, x2 = 0xFFFFFFFFu;
     uint64_t rn1 = r;
     if (t + 1 < wn) {
-      wn1 = posof(t + 1);
-      if (test_admit) rn1 = ws.recvs[wn1];
+      const uint32_t xn = posof(t + 1);
+      wn1 = ws.wl[xn];
+      if (test_admit) rn1 = hdrof(xn);
     }
     const uint32_t cur_now = cur;
     if (t + 1 < wn) {
@@ -280,8 +278,6 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     MM_PHASE(0);
 
     // P1 -------------------------------------------------------------------
-    stage_side<NT>(a.M, e, nm, mres, mpb, ws.msgs, tid);
-    stage_side<NT>(a.R, e, nr, rres, rpb, ws.recvs, tid);
     for (uint32_t s = tid; s < H / 2; s += NT) reinterpret_cast<uint32_t*>(ws.table)[s] = 0xFFFFFFFFu;
     for (int64_t k = tid; k < (nm + 31) / 32; k += NT) ws.matched[k] = 0u;
     if (tid == 0) {
@@ -293,28 +289,45 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     // P2 -------------------------------------------------------------------
     // insert message tuples; the CAS winner of a slot takes the next dense
     // tuple id and initialises the tuple's entries (no separate id pass)
-    for (int64_t j = tid; j < nm; j += NT) {
-      const uint64_t h = ws.msgs[j];
+    for (int64_t j0 = tid; j0 < nm; j0 += 4 * NT) {
+     uint64_t hv[4];
+#pragma unroll
+     for (int u = 0; u < 4; u++) {  // read once from HBM (not staged), four loads in flight
+       const int64_t j = j0 + (int64_t)u * NT;
+       hv[u] = j < nm ? a.M.hdr(e, j, mres, mpb) : 0ull;
+     }
+#pragma unroll
+     for (int u = 0; u < 4; u++) {
+      const int64_t j = j0 + (int64_t)u * NT;
+      if (j >= nm) break;
+      const uint64_t h = hv[u];
       uint32_t s = slot_hash(h) & hmask;
+      uint32_t id;
       while (true) {
         uint16_t o = ws.table[s];
         if (o == kEmpty16) {
-          o = cas16(&ws.table[s], kEmpty16, (uint16_t)j);
-          if (o == kEmpty16) {
-            const uint32_t id = atomicAdd(&sh_K, 1u);
-            ws.slot_id[s] = (uint16_t)id;
+          o = cas16(&ws.table[s], kEmpty16, kPending16);
+          if (o == kEmpty16) {  // this message opens the tuple
+            id = atomicAdd(&sh_K, 1u);
             ws.keyhdr[id] = h;
 #pragma unroll
             for (int q = 0; q < 8; q++) ws.pcnt[q * ws.mcap + id] = 0;
             ws.key_c[id] = 0;
             ws.key_cur[id] = 0;
+            __threadfence_block();
+            *reinterpret_cast<volatile uint16_t*>(&ws.table[s]) = (uint16_t)id;
             break;
           }
         }
-        if (ws.msgs[o] == h) break;
+        while (o == kPending16) o = *reinterpret_cast<volatile uint16_t*>(&ws.table[s]);
+        if (ws.keyhdr[o] == h) {
+          id = o;
+          break;
+        }
         s = (s + 1) & hmask;
       }
-      ws.msg_key[j] = (uint16_t)s;
+      ws.msg_key[j] = (uint16_t)id;
+     }
     }
     __syncthreads();
     MM_PHASE(2);
@@ -323,31 +336,38 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     const uint32_t K = sh_K;
     MM_PHASE(3);
     // P4 -------------------------------------------------------------------
-    for (int64_t j = tid; j < nm; j += NT) {
-      const uint16_t id = ws.slot_id[ws.msg_key[j]];
-      ws.msg_key[j] = id;
-      inc16(&ws.pcnt[(int64_t)((j * 4) / nm) * ws.mcap + id]);
-    }
-    for (int64_t i = tid; i < nr; i += NT) {
-      const uint64_t h = ws.recvs[i];
-      uint16_t rk;
-      if (wildcard_mask(h) != ~0ull) {
-        rk = kWild;
-      } else {
-        rk = kNone;
-        uint32_t s = slot_hash(h) & hmask;
-        while (true) {
-          const uint16_t o = ws.table[s];
-          if (o == kEmpty16) break;
-          if (ws.msgs[o] == h) {
-            rk = ws.slot_id[s];
-            break;
-          }
-          s = (s + 1) & hmask;
-        }
-        if (rk != kNone) inc16(&ws.pcnt[(4 + (int64_t)((i * 4) / nr)) * ws.mcap + rk]);
+    for (int64_t j = tid; j < nm; j += NT) inc16(&ws.pcnt[(int64_t)((j * 4) / nm) * ws.mcap + ws.msg_key[j]]);
+    for (int64_t i0 = tid; i0 < nr; i0 += 4 * NT) {
+      uint64_t hv[4];
+#pragma unroll
+      for (int u = 0; u < 4; u++) {  // four independent HBM loads in flight
+        const int64_t i = i0 + (int64_t)u * NT;
+        hv[u] = i < nr ? a.R.hdr(e, i, rres, rpb) : 0ull;
       }
-      ws.recv_key[i] = rk;
+#pragma unroll
+      for (int u = 0; u < 4; u++) {
+        const int64_t i = i0 + (int64_t)u * NT;
+        if (i >= nr) break;
+        const uint64_t h = hv[u];
+        uint16_t rk;
+        if (wildcard_mask(h) != ~0ull) {
+          rk = kWild;
+        } else {
+          rk = kNone;
+          uint32_t s = slot_hash(h) & hmask;
+          while (true) {
+            const uint16_t o = ws.table[s];
+            if (o == kEmpty16) break;
+            if (ws.keyhdr[o] == h) {
+              rk = o;
+              break;
+            }
+            s = (s + 1) & hmask;
+          }
+          if (rk != kNone) inc16(&ws.pcnt[(4 + (int64_t)((i * 4) / nr)) * ws.mcap + rk]);
+        }
+        ws.recv_key[i] = rk;
+      }
     }
     __syncthreads();
     MM_PHASE(4);
@@ -387,11 +407,18 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       uint32_t wt;
       uint32_t wp = block_excl_scan<uint32_t>(wc, scan_sm, &wt);
       for (uint32_t i = i0; i < i1 && wc; i++)
-        if (ws.recv_key[i] == kWild) ws.wl[wp++] = (uint16_t)i;
+        if (ws.recv_key[i] == kWild) {
+          if (wp < L.wcap) ws.whdr[wp] = a.R.hdr(e, i, rres, rpb);
+          ws.wl[wp++] = (uint16_t)i;
+        }
       if (tid == 0) sh_W = wt;
     }
     __syncthreads();
     const uint32_t W = sh_W;
+    // header of the x-th wildcard (staged for the first wcap of them)
+    auto hdrof = [&](uint32_t x) -> uint64_t {
+      return x < L.wcap ? ws.whdr[x] : a.R.hdr(e, ws.wl[x], rres, rpb);
+    };
     MM_PHASE(5);
     // P6 -------------------------------------------------------------------
     // warps 0-3 place the four quarters of the messages, warps 4-7 the four
@@ -427,7 +454,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       if (tid == 0) sh_types = 0;
       __syncthreads();
       for (uint32_t x = tid; x < W; x += NT) {
-        const uint64_t r = ws.recvs[ws.wl[x]];
+        const uint64_t r = hdrof(x);
         const uint32_t code = ((uint32_t)r == MM_ANY_SOURCE ? 1u : 0u) |
                               (((uint32_t)(r >> 32) & 0xFFFFu) == MM_ANY_TAG ? 2u : 0u);
         atomicOr(&sh_types, 1u << code);
@@ -439,8 +466,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       // parallel phases of co-resident CTAs (B300_MICROARCH.md, arbiter)
       if (K <= 32) {
         if (warp == NT / 32 - 1)
-          register_chain(ws, K, [](uint32_t l) { return l; }, W, [&](uint32_t t) { return (uint32_t)ws.wl[t]; }, true,
-                         lane);
+          register_chain(ws, K, [](uint32_t l) { return l; }, W, [](uint32_t t) { return t; }, hdrof, true, lane);
         MM_PHASE(11);
 #ifdef MM_PHASE_TIMING
         if (tid == 0) atomicAdd(&g_phase_cycles[13], 1ull);
@@ -452,54 +478,49 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         const uint32_t code = __ffs(types) - 1;
         const uint64_t gmsk = (code & 1 ? ~0xFFFFFFFFull : ~0ull) & (code & 2 ? ~(0xFFFFull << 32) : ~0ull);
         for (uint32_t s2 = tid; s2 < H / 2; s2 += NT) reinterpret_cast<uint32_t*>(ws.table)[s2] = 0xFFFFFFFFu;
+        if (tid == 0) sh_G = 0;
         __syncthreads();
+        // group table: entry = representative tuple; the CAS winner takes the
+        // next group id and publishes it through key_grp[representative]
         for (uint32_t k = tid; k < K; k += NT) {
           const uint64_t gk = ws.keyhdr[k] & gmsk;
           uint32_t sl = slot_hash(gk) & hmask;
+          uint32_t g;
           while (true) {
             uint16_t o = ws.table[sl];
             if (o == kEmpty16) {
-              o = cas16(&ws.table[sl], kEmpty16, (uint16_t)k);
-              if (o == kEmpty16) break;
+              o = cas16(&ws.table[sl], kEmpty16, kPending16);
+              if (o == kEmpty16) {
+                g = atomicAdd(&sh_G, 1u);
+                ws.key_grp[k] = (uint16_t)g;
+                ws.g_cnt[g] = 0;
+                ws.gw_cnt[g] = 0;
+                __threadfence_block();
+                *reinterpret_cast<volatile uint16_t*>(&ws.table[sl]) = (uint16_t)k;
+                break;
+              }
             }
-            if ((ws.keyhdr[o] & gmsk) == gk) break;
+            while (o == kPending16) o = *reinterpret_cast<volatile uint16_t*>(&ws.table[sl]);
+            if ((ws.keyhdr[o] & gmsk) == gk) {
+              g = *reinterpret_cast<volatile uint16_t*>(&ws.key_grp[o]);
+              ws.key_grp[k] = (uint16_t)g;
+              break;
+            }
             sl = (sl + 1) & hmask;
           }
-          ws.key_grp[k] = (uint16_t)sl;
-        }
-        __syncthreads();
-        {
-          const uint32_t per = (H + NT - 1) / NT;
-          const uint32_t s0 = min(H, tid * per), s1 = min(H, s0 + per);
-          uint32_t c = 0;
-          for (uint32_t q = s0; q < s1; q++) c += ws.table[q] != kEmpty16;
-          uint32_t tot;
-          uint32_t id = block_excl_scan<uint32_t>(c, scan_sm, &tot);
-          for (uint32_t q = s0; q < s1; q++)
-            if (ws.table[q] != kEmpty16) {
-              ws.slot_id[q] = (uint16_t)id;
-              ws.g_cnt[id] = 0;
-              ws.gw_cnt[id] = 0;
-              id++;
-            }
-          if (tid == 0) sh_G = tot;
         }
         __syncthreads();
         const uint32_t G = sh_G;
-        for (uint32_t k = tid; k < K; k += NT) {
-          const uint16_t g = ws.slot_id[ws.key_grp[k]];
-          ws.key_grp[k] = g;
-          inc16(&ws.g_cnt[g]);
-        }
+        for (uint32_t k = tid; k < K; k += NT) inc16(&ws.g_cnt[ws.key_grp[k]]);
         for (uint32_t x = tid; x < W; x += NT) {
-          const uint64_t rg = ws.recvs[ws.wl[x]] & gmsk;
+          const uint64_t rg = hdrof(x) & gmsk;
           uint32_t sl = slot_hash(rg) & hmask;
           uint16_t g = kNone;
           while (true) {
             const uint16_t o = ws.table[sl];
             if (o == kEmpty16) break;
             if ((ws.keyhdr[o] & gmsk) == rg) {
-              g = ws.slot_id[sl];
+              g = ws.key_grp[o];
               break;
             }
             sl = (sl + 1) & hmask;
@@ -548,11 +569,12 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             // cursor and claim count in registers, so one wildcard costs a
             // cursor step, one head read and one redux.
             register_chain(ws, kn, [&](uint32_t l) { return (uint32_t)ws.g_keys[ks0 + l]; }, wn,
-                           [&](uint32_t t) { return (uint32_t)ws.wl[ws.gw_list[ws0 + t]]; }, false, lane);
+                           [&](uint32_t t) { return (uint32_t)ws.gw_list[ws0 + t]; }, hdrof, false, lane);
           } else {
             for (uint32_t t = 0; t < wn; t++) {
-              const uint32_t w = ws.wl[ws.gw_list[ws0 + t]];
-              const uint64_t r = ws.recvs[w];
+              const uint32_t xg = ws.gw_list[ws0 + t];
+              const uint32_t w = ws.wl[xg];
+              const uint64_t r = hdrof(xg);
               resolve_wildcard(ws, w, r, wildcard_mask(r), kn,
                                [&](uint32_t c0) { return (uint32_t)ws.g_keys[ks0 + c0]; }, lane);
             }
@@ -561,7 +583,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       } else if (warp == NT / 32 - 1) {
         for (uint32_t x = 0; x < W; x++) {
           const uint32_t w = ws.wl[x];
-          const uint64_t r = ws.recvs[w];
+          const uint64_t r = hdrof(x);
           resolve_wildcard(ws, w, r, wildcard_mask(r), K, [](uint32_t c0) { return c0; }, lane);
         }
       }
@@ -596,10 +618,11 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         }
         const uint32_t um = (valid && res == kNone) ? 1u : 0u;
         nmatch += (valid && res != kNone) ? 1u : 0u;
+        const uint64_t rh = um ? a.R.hdr(e, i, rres, rpb) : 0ull;
         uint32_t tot;
         const uint32_t pos = wr + block_excl_scan<uint32_t>(um, scan_sm, &tot);  // syncs: reads precede writes
         if (um) {
-          qrh[pos] = ws.recvs[i];
+          qrh[pos] = rh;
           qrc[pos] = rc;
         }
         wr += tot;
@@ -619,11 +642,15 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         const int64_t j = b0 + tid;
         const bool keep = j < nm && !((ws.matched[j >> 5] >> (j & 31)) & 1u);
         int64_t c = 0;
-        if (keep) c = a.M.cookie(e, j, mres, mpb);
-        uint32_t tot;
+        uint64_t h = 0;
+        if (keep) {
+          c = a.M.cookie(e, j, mres, mpb);
+          h = a.M.hdr(e, j, mres, mpb);
+        }
+        uint32_t tot;  // (the scan's barriers order these reads before the in-place writes)
         const uint32_t pos = wm + block_excl_scan<uint32_t>(keep ? 1u : 0u, scan_sm, &tot);
         if (keep) {
-          qmh[pos] = ws.msgs[j];
+          qmh[pos] = h;
           qmc[pos] = c;
         }
         wm += tot;
@@ -652,11 +679,10 @@ FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
     return o;
   };
   auto r16 = [](int64_t b) { return (b + 15) / 16 * 16; };
-  L.msgs = take(8 * mcap);
-  L.recvs = take(8 * rcap);
+  L.wcap = (uint32_t)((rcap + 7) / 8 > 32 ? (rcap + 7) / 8 : 32);  // wildcard headers kept on chip
+  L.whdr = take(8 * (int64_t)L.wcap);
   L.keyhdr = take(8 * mcap);
   L.table = take(2 * H);
-  L.slot_id = take(2 * H);
   L.key_cnt = take(2 * mcap);
   L.key_start = take(2 * mcap);
   L.key_rcnt = take(2 * mcap);

@@ -10,6 +10,7 @@ namespace mm {
 constexpr uint16_t kWild = 0xFFFEu;
 constexpr uint16_t kNone = 0xFFFFu;
 constexpr uint16_t kEmpty16 = 0xFFFFu;
+constexpr uint16_t kPending16 = 0xFFFEu;  // slot claimed, id not yet published
 
 // Slot of a tuple in an on-chip hash table: multiply-shift of the 64-bit word
 // (a few instructions; the tables are small and private to one CTA).
