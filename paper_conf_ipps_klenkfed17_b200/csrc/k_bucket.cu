@@ -162,12 +162,11 @@ struct BucketSmem {
   uint16_t key[kBucketCap];      // tuple id | kNone
   uint16_t rank[kBucketCap];     // rank among the equal tuples of the element's side
   uint16_t table[kBucketH];      // slot -> representative message (element index)
-  uint16_t slot_id[kBucketH];    // slot -> tuple id
   uint16_t cnt_m[kBucketCap];    // messages per tuple
   uint16_t start_m[kBucketCap];  // start of the tuple in by_key
   uint16_t cnt_r[kBucketCap];    // receives per tuple
   uint16_t by_key[kBucketCap];   // messages grouped by tuple, in rank order (element index)
-  uint16_t pcnt[ORDERED ? 8 : 2][kBucketCap];  // per-quarter counts / running ranks (msgs, then receives)
+  uint16_t pcnt[ORDERED ? 4 : 2][kBucketCap];  // per-half counts / running ranks (msgs, then receives)
   uint32_t scan[kBucketThreads / 32 + 1];
   uint32_t K;
   uint32_t matched;
@@ -177,7 +176,8 @@ template <bool ORDERED>
 __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   BucketSmem<ORDERED>& sm = *reinterpret_cast<BucketSmem<ORDERED>*>(smem_raw);
-  constexpr int RROW = ORDERED ? 4 : 1;  // first pcnt row of the receive side
+  constexpr int QN = ORDERED ? 2 : 1;  // ordered: each side placed in two halves by two warps
+  constexpr int RROW = QN;             // first pcnt row of the receive side
   constexpr int NT = kBucketThreads;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t lt = lanemask_lt();
@@ -209,7 +209,9 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
     sm.K = 0;
   }
   __syncthreads();
-  // message tuples into the hash table; the CAS winner takes the next dense id
+  // message tuples into the hash table (slot -> representative element); the
+  // CAS winner takes the next dense id and records it in rank[representative]
+  // (rank is only filled later, by the ranking step)
   for (uint32_t e = nr + tid; e < n; e += NT) {
     const uint64_t h = sm.hdr[e];
     uint32_t s = slot_hash(h) & hmask;
@@ -219,25 +221,26 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
         o = cas16(&sm.table[s], kEmpty16, (uint16_t)e);
         if (o == kEmpty16) {
           const uint32_t id = atomicAdd(&sm.K, 1u);
-          sm.slot_id[s] = (uint16_t)id;
+          sm.rank[e] = (uint16_t)id;
 #pragma unroll
-          for (int q = 0; q < (ORDERED ? 8 : 2); q++) sm.pcnt[q][id] = 0;
+          for (int q = 0; q < 2 * QN; q++) sm.pcnt[q][id] = 0;
+          o = (uint16_t)e;
           break;
         }
       }
       if (sm.hdr[o] == h) break;
       s = (s + 1) & hmask;
     }
-    sm.key[e] = (uint16_t)s;
+    sm.key[e] = (uint16_t)(s);  // slot for now
   }
   __syncthreads();
   const uint32_t K = sm.K;
-  // tuple ids; quarter counts (ordered) or plain counts (unordered, row 0/4)
+  // tuple ids; per-half counts (ordered) or plain counts (unordered)
   for (uint32_t e = tid; e < n; e += NT) {
     uint16_t k;
     const bool is_msg = e >= nr;
     if (is_msg) {
-      k = sm.slot_id[sm.key[e]];
+      k = sm.rank[sm.table[sm.key[e]]];
     } else {
       const uint64_t h = sm.hdr[e];
       uint32_t s = slot_hash(h) & hmask;
@@ -246,7 +249,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
         const uint16_t o = sm.table[s];
         if (o == kEmpty16) break;
         if (sm.hdr[o] == h) {
-          k = sm.slot_id[s];
+          k = sm.rank[o];
           break;
         }
         s = (s + 1) & hmask;
@@ -255,7 +258,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
     sm.key[e] = k;
     if (k != kNone) {
       const uint32_t side_n = is_msg ? nm : nr, x = is_msg ? e - nr : e;
-      const uint32_t q = ORDERED ? (uint32_t)(((uint64_t)x * 4) / side_n) : 0u;
+      const uint32_t q = ORDERED ? (uint32_t)(((uint64_t)x * QN) / side_n) : 0u;
       inc16(&sm.pcnt[(is_msg ? 0 : RROW) + q][k]);
     }
   }
@@ -267,7 +270,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
     for (uint32_t k = k0; k < k1; k++) {
       uint32_t rm = 0, rr = 0;
 #pragma unroll
-      for (int q = 0; q < (ORDERED ? 4 : 1); q++) {
+      for (int q = 0; q < QN; q++) {
         const uint32_t x = sm.pcnt[q][k], y = sm.pcnt[RROW + q][k];
         sm.pcnt[q][k] = (uint16_t)rm;
         sm.pcnt[RROW + q][k] = (uint16_t)rr;
@@ -287,21 +290,20 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
   }
   __syncthreads();
   // ranks
-  if (ORDERED) {
-    const bool msg_side = warp < 4;
-    const int q = warp & 3;
+  if (ORDERED && warp < 2 * QN) {
+    const bool msg_side = warp < QN;
+    const int q = warp % QN;
     const uint32_t side_n = msg_side ? nm : nr, base = msg_side ? nr : 0;
-    const int64_t x0 = ((int64_t)side_n * q + 3) / 4, x1 = ((int64_t)side_n * (q + 1) + 3) / 4;
+    const int64_t x0 = ((int64_t)side_n * q + QN - 1) / QN, x1 = ((int64_t)side_n * (q + 1) + QN - 1) / QN;
     place_in_order(
-        x1 - x0, [&](int64_t x) { return (uint32_t)sm.key[base + x0 + x]; }, msg_side ? sm.start_m : sm.start_m,
-        sm.pcnt[ORDERED ? warp : 0],
+        x1 - x0, [&](int64_t x) { return (uint32_t)sm.key[base + x0 + x]; }, sm.start_m, sm.pcnt[warp],
         [&](int64_t x, uint32_t k, uint32_t r, uint32_t slot) {
           const uint32_t e = base + (uint32_t)(x0 + x);
           sm.rank[e] = (uint16_t)r;
           if (msg_side) sm.by_key[slot] = (uint16_t)e;
         },
         lane, lt, K);
-  } else {
+  } else if (!ORDERED) {
     for (uint32_t e = tid; e < n; e += NT) {
       const uint16_t k = sm.key[e];
       if (k == kNone) continue;
