@@ -1,0 +1,19 @@
+# Full round evidence: gpu tests, smoke, bench (with cpu baseline), ncu launch list, ncu --set full of the top kernels.
+# usage: bash tools/gpu_round.sh <tag>
+cd $GRAFT_REPO_ROOT
+TAG=${1:-x}
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build_$TAG.log 2>&1 || { tail -20 gpurun_out/build_$TAG.log; exit 1; }
+timeout 1500 python -m pytest tests -m gpu -q --maxfail=5 -p no:cacheprovider > gpurun_out/pytest_$TAG.log 2>&1; tail -2 gpurun_out/pytest_$TAG.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -1
+timeout 900 python bench.py > gpurun_out/bench_$TAG.log 2>&1; tail -1 gpurun_out/bench_$TAG.log | python -c "
+import json,sys; d=json.loads(sys.stdin.read())
+print('clocks', d['clocks'])
+for k,v in d['levels'].items(): print(k, round(v['value']/1e9,3), 'Gm/s', round(v['ms_per_step'],3), 'ms kernel', round(v['roofline']['kernel_ms'],3), 'frac', round(v['roofline']['frac'],4))"
+timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv \
+    --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline > gpurun_out/ncu_launch_$TAG.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_mpi_fifo|k_mpi_matrix" -s 6 -c 2 -o gpurun_out/prof_mpi_$TAG \
+    python bench.py --steps 1 --warmup 3 --levels mpi,mpi_matrix --no-cpu-baseline > gpurun_out/ncu_mpi_$TAG.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_part_scatter|k_bucket_pair|k_part_hist|k_bucket_bounds" -s 20 -c 8 -o gpurun_out/prof_flat_$TAG \
+    python bench.py --steps 1 --warmup 3 --levels ordered,unordered --no-cpu-baseline > gpurun_out/ncu_flat_$TAG.log 2>&1
+ls gpurun_out | grep $TAG
