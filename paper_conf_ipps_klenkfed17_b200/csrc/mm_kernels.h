@@ -27,9 +27,8 @@ struct MpiArgs {
 // Key-FIFO engine workspace (byte offsets inside one CTA's workspace).
 constexpr int64_t kFifoSmemMax = 100 * 1024;
 struct FifoLayout {
-  int64_t whdr, keyhdr, table, key_cnt, key_start, key_rcnt, key_rstart, key_c, key_cur, msg_key, by_key,
-      wlog, recv_key, recv_e, rby_key, recv_res, wl, matched, key_grp, g_cnt, g_start, g_keys, gw_cnt, gw_start,
-      w_grp, gw_list, pcnt, mcap;
+  int64_t whdr, keyhdr, table, key_cnt, key_start, key_rcnt, key_rstart, key_c, msg_key, by_key,
+      wlog, recv_key, recv_e, rby_key, recv_res, wl, matched, pcnt, gnext, gfirst, gwc, w_grp, mcap;
   int64_t total;
   uint32_t H;
   uint32_t wcap;
