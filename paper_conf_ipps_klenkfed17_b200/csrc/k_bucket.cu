@@ -54,6 +54,10 @@ struct BDigit {
     const uint32_t b = FIRST ? bucket_of(snap.hdr(k), nb) : (uint32_t)(bi[k] >> 32);
     return (b >> shift) & (uint32_t)dmask;
   }
+  // the same digit from the element's loaded payload (BMove::load)
+  __device__ __forceinline__ uint32_t of_payload(int64_t, uint64_t a, uint64_t b) const {
+    return ((uint32_t)(b >> 32) >> shift) & (uint32_t)dmask;
+  }
 };
 template <bool FIRST>
 struct BMove {
@@ -79,15 +83,36 @@ struct BMove {
 };
 
 // off[b] = first position of bucket b in the bucket-sorted array (b in 0..B).
+// Four consecutive elements per thread, read as two 16-byte vectors.
 __global__ void k_bucket_bounds(const uint64_t* bi, int64_t n, int nb, uint32_t* off) {
   const uint32_t B = 1u << nb;
-  for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < n; p += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t b = (uint32_t)(bi[p] >> 32);
-    const uint32_t prev = p == 0 ? 0xFFFFFFFFu : (uint32_t)(bi[p - 1] >> 32);
-    if (b != prev)
-      for (uint32_t x = prev + 1; x <= b; x++) off[x] = (uint32_t)p;  // (prev+1 wraps to 0 at p == 0)
-    if (p == n - 1)
-      for (uint32_t x = b + 1; x <= B; x++) off[x] = (uint32_t)n;
+  const int64_t nq = (n + 3) / 4;
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t p0 = q * 4;
+    uint64_t v[4];
+    if (p0 + 4 <= n) {
+      const ulonglong2 x = reinterpret_cast<const ulonglong2*>(bi + p0)[0];
+      const ulonglong2 y = reinterpret_cast<const ulonglong2*>(bi + p0)[1];
+      v[0] = x.x;
+      v[1] = x.y;
+      v[2] = y.x;
+      v[3] = y.y;
+    } else {
+#pragma unroll
+      for (int j = 0; j < 4; j++) v[j] = p0 + j < n ? bi[p0 + j] : 0ull;
+    }
+    uint32_t prev = p0 == 0 ? 0xFFFFFFFFu : (uint32_t)(bi[p0 - 1] >> 32);
+#pragma unroll
+    for (int j = 0; j < 4; j++) {
+      const int64_t p = p0 + j;
+      if (p >= n) break;
+      const uint32_t b = (uint32_t)(v[j] >> 32);
+      if (b != prev)
+        for (uint32_t x = prev + 1; x <= b; x++) off[x] = (uint32_t)p;  // (prev+1 wraps to 0 at p == 0)
+      if (p == n - 1)
+        for (uint32_t x = b + 1; x <= B; x++) off[x] = (uint32_t)n;
+      prev = b;
+    }
   }
 }
 __global__ void k_fill_u32(uint32_t* a, int64_t n, uint32_t v) {
@@ -133,7 +158,7 @@ static cudaError_t partition_side(const SnapRead& snap, int64_t n, int nb, uint6
     if (err != cudaSuccess) return err;
   }
   count_launch();
-  k_bucket_bounds<<<grid_cap(n, 256), 256, 0, st>>>(ib[cur], n, nb, off);
+  k_bucket_bounds<<<grid_cap((n + 3) / 4, 256), 256, 0, st>>>(ib[cur], n, nb, off);
   *out_h = hb[cur];
   *out_i = ib[cur];
   return cudaGetLastError();

@@ -93,6 +93,9 @@ struct DigitOf {
   const uint64_t* key;
   int shift;
   __device__ __forceinline__ uint32_t operator()(int64_t k) const { return (uint32_t)(key[k] >> shift) & 255u; }
+  __device__ __forceinline__ uint32_t of_payload(int64_t, uint64_t a, uint64_t) const {
+    return (uint32_t)(a >> shift) & 255u;
+  }
 };
 struct MoveKV {
   const uint64_t* ki;
@@ -394,6 +397,10 @@ struct OwnerOf {
   __device__ __forceinline__ uint32_t operator()(int64_t k) const {
     if (by == 1) return (uint32_t)(a[k] >> 40);
     return (uint32_t)(((unsigned long long)header_hash(a[k]) * (unsigned)world) >> 32);
+  }
+  __device__ __forceinline__ uint32_t of_payload(int64_t, uint64_t x, uint64_t) const {
+    if (by == 1) return (uint32_t)(x >> 40);
+    return (uint32_t)(((unsigned long long)header_hash(x) * (unsigned)world) >> 32);
   }
 };
 struct MoveRoute {

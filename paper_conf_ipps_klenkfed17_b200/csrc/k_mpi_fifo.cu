@@ -206,22 +206,26 @@ __device__ __forceinline__ void resolve_wildcard(const FifoWs& ws, uint32_t x, u
 }
 
 // A chain of wildcard receives over at most 32 candidate tuples, one tuple per
-// lane (own, k) with its cursor and claim count in registers.  next() yields
-// the wildcards (indices into wl) in posting order, kNone32 at the end; it is
-// warp-uniform.  The head a lane offers at step t is list_k[e_k(w_t) + c];
-// e_k(w_t) does not depend on the chain and c grows by one only when the lane
-// wins, so the three candidates list_k[e + c], list_k[e + c + 1],
-// list_k[e + c + 2] of the NEXT step are loaded while the current step
+// lane (own, k) with its cursor and claim count in registers.  gen(x, w, r)
+// yields the wildcards in posting order (x = index into wl, w = posting
+// position, r = header when test_admit) and false at the end; it is
+// warp-uniform and serves positions from registers (a chunk of 32 loaded at a
+// time).  The head a lane offers at step t is list_k[e_k(w_t) + c]; e_k(w_t)
+// does not depend on the chain (the cursor keeps the position of the next
+// exact receive of k in a register, so it usually moves without a load) and c
+// grows by one only when the lane wins, so the window list_k[e + c .. e + c + 3]
+// of the NEXT step is formed (mostly from registers) while the current step
 // resolves: the critical path of a wildcard is one redux.sync.min and a
-// select, no shared-memory load.
+// select.
 // test_admit: wildcards may differ, so each lane tests admission with the
 // masked XOR; otherwise every wildcard admits every candidate (a group).
-template <class NextF, class HdrF>
-__device__ __forceinline__ void register_chain(const FifoWs& ws, bool own, uint32_t k, NextF next, HdrF hdrof,
-                                               bool test_admit, int lane) {
-  uint32_t x = next();
-  if (x == kNone32) return;
-  uint32_t cur = 0, c = 0, rs = 0, rc = 0, st = 0, cnt = 0;
+template <class GenF>
+__device__ __forceinline__ void register_chain(const FifoWs& ws, bool own, uint32_t k, GenF gen, bool test_admit,
+                                               int lane) {
+  uint32_t x, w;
+  uint64_t r;
+  if (!gen(x, w, r)) return;
+  uint32_t cur = 0, c = 0, rs = 0, rc = 0, st = 0, cnt = 0, npos = 0xFFFFFFFFu;
   uint64_t kh = 0;
   if (own) {
     rs = ws.key_rstart[k];
@@ -229,29 +233,42 @@ __device__ __forceinline__ void register_chain(const FifoWs& ws, bool own, uint3
     st = ws.key_start[k];
     cnt = ws.key_cnt[k];
     kh = ws.keyhdr[k];
+    if (rc) npos = ws.rby_key[rs];
   }
   auto head_at = [&](uint32_t i) { return (own && i < cnt) ? (uint32_t)ws.by_key[st + i] : 0xFFFFFFFFu; };
-  // cursor: exact receives of k posted before w (monotone in w)
+  // cursor: exact receives of k posted before w (monotone in w); npos = the
+  // posting position of the next one
   auto advance = [&](uint32_t w) {
-    if (own)
-      while (cur < rc && ws.rby_key[rs + cur] < w) cur++;
+    while (npos < w) {
+      cur++;
+      npos = cur < rc ? (uint32_t)ws.rby_key[rs + cur] : 0xFFFFFFFFu;
+    }
   };
-  uint32_t w = ws.wl[x];
-  uint64_t r = test_admit ? hdrof(x) : 0ull;
   advance(w);
   uint32_t h0 = head_at(cur + c), h1 = head_at(cur + c + 1), h2 = head_at(cur + c + 2);
   while (true) {
-    // loads for the next step, independent of this step's outcome
-    const uint32_t xn = next();
-    uint32_t wn1 = w, x0 = 0xFFFFFFFFu, x1 = 0xFFFFFFFFu, x2 = 0xFFFFFFFFu;
-    uint64_t rn1 = r;
-    if (xn != kNone32) {
-      wn1 = ws.wl[xn];
-      if (test_admit) rn1 = hdrof(xn);
-      advance(wn1);
-      x0 = head_at(cur + c);
-      x1 = head_at(cur + c + 1);
-      x2 = head_at(cur + c + 2);
+    // the next step's window, independent of this step's outcome
+    uint32_t xn, wn;
+    uint64_t rn;
+    const bool more = gen(xn, wn, rn);
+    uint32_t y0 = h0, y1 = h1, y2 = h2, y3 = 0xFFFFFFFFu;
+    if (more) {
+      const uint32_t cur0 = cur;
+      advance(wn);
+      const uint32_t d = cur - cur0, b = cur + c;
+      if (d == 0) {
+        y3 = head_at(b + 3);
+      } else if (d == 1) {
+        y0 = h1;
+        y1 = h2;
+        y2 = head_at(b + 2);
+        y3 = head_at(b + 3);
+      } else {
+        y0 = head_at(b);
+        y1 = head_at(b + 1);
+        y2 = head_at(b + 2);
+        y3 = head_at(b + 3);
+      }
     }
     uint32_t cand = h0;
     if (test_admit && ((kh ^ r) & wildcard_mask(r)) != 0) cand = 0xFFFFFFFFu;
@@ -262,14 +279,14 @@ __device__ __forceinline__ void register_chain(const FifoWs& ws, bool own, uint3
       c++;
     }
     if (lane == 0) ws.recv_res[x] = win == 0xFFFFFFFFu ? kNone : (uint16_t)win;
-    if (xn == kNone32) break;
+    if (!more) break;
     // next step's heads: list_k[cur' + c'] with c' = c (+1 if won)
-    h0 = won ? x1 : x0;
-    h1 = won ? x2 : x1;
-    h2 = won ? head_at(cur + c + 2) : x2;  // rare third load only after a win
+    h0 = won ? y1 : y0;
+    h1 = won ? y2 : y1;
+    h2 = won ? y3 : y2;
     x = xn;
-    w = wn1;
-    r = rn1;
+    w = wn;
+    r = rn;
   }
   if (own) ws.key_c[k] = (uint16_t)c;
 }
@@ -501,9 +518,22 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     if (W > 0) {
       if (K <= 32) {
         if (warp == NW - 1) {
-          uint32_t t = 0;
-          register_chain(
-              ws, lane < K, (uint32_t)lane, [&]() { return t < W ? t++ : kNone32; }, hdrof, true, lane);
+          uint32_t t = 0, wv = 0;
+          uint64_t rv = 0;
+          auto gen = [&](uint32_t& xo, uint32_t& wo, uint64_t& ro) -> bool {
+            if (t >= W) return false;
+            if ((t & 31) == 0) {  // next chunk of 32 wildcards into registers
+              const uint32_t y = t + lane;
+              wv = y < W ? ws.wl[y] : 0u;
+              rv = y < W ? hdrof(y) : 0ull;
+            }
+            xo = t;
+            wo = __shfl_sync(kFull, wv, t & 31);
+            ro = __shfl_sync(kFull, rv, t & 31);
+            t++;
+            return true;
+          };
+          register_chain(ws, lane < (int)K, (uint32_t)lane, gen, true, lane);
         }
         MM_PHASE(11);
 #ifdef MM_PHASE_TIMING
@@ -588,24 +618,32 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             // the group's wildcards in posting order, from its first one
             uint32_t left = ws.gwc[gg];
             uint32_t cb = b, cm = __ballot_sync(kFull, g == gg) & (~0u << l);
-            auto next = [&]() -> uint32_t {
-              if (left == 0) return kNone32;
-              while (cm == 0) {
+            uint32_t wv = g == gg ? ws.wl[x] : 0u;
+            auto gen = [&](uint32_t& xo, uint32_t& wo, uint64_t& ro) -> bool {
+              if (left == 0) return false;
+              while (cm == 0) {  // next chunk holding wildcards of the group
                 cb += 32;
                 const uint32_t y = cb + lane;
-                cm = __ballot_sync(kFull, y < W && ws.w_grp[y] == gg);
+                const bool in = y < W && ws.w_grp[y] == gg;
+                cm = __ballot_sync(kFull, in);
+                wv = in ? ws.wl[y] : 0u;
               }
-              const uint32_t xx = cb + __ffs(cm) - 1;
+              const int bit = __ffs(cm) - 1;
               cm &= cm - 1;
               left--;
-              return xx;
+              xo = cb + bit;
+              wo = __shfl_sync(kFull, wv, bit);
+              ro = 0;
+              return true;
             };
             if (kn <= 32) {
-              register_chain(ws, lane < (int)kn, mine, next, hdrof, false, lane);
+              register_chain(ws, lane < (int)kn, mine, gen, false, lane);
             } else {  // a group of more than 32 tuples: scan every tuple, admission tested
-              for (uint32_t xx = next(); xx != kNone32; xx = next()) {
+              uint32_t xx, ww;
+              uint64_t rr;
+              while (gen(xx, ww, rr)) {
                 const uint64_t r = hdrof(xx);
-                resolve_wildcard(ws, xx, ws.wl[xx], r, wildcard_mask(r), K, [](uint32_t c0) { return c0; }, lane);
+                resolve_wildcard(ws, xx, ww, r, wildcard_mask(r), K, [](uint32_t c0) { return c0; }, lane);
               }
             }
           }

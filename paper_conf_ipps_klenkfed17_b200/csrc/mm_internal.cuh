@@ -215,11 +215,16 @@ __global__ void __launch_bounds__(kPartThreads) k_part_hist(BucketF bucket, int6
   for (int b = threadIdx.x; b < kPartMaxBuckets; b += blockDim.x) h[b] = 0;
   __syncthreads();
   const int64_t base = (int64_t)blockIdx.x * kPartTile;
-#pragma unroll 4
-  for (int i = threadIdx.x; i < kPartTile; i += kPartThreads) {
-    int64_t k = base + i;
-    if (k < n) atomicAdd(&h[bucket(k)], 1u);
+  constexpr int kPer = kPartTile / kPartThreads;  // 16 elements per thread, all loads in flight
+  uint32_t bk[kPer];
+#pragma unroll
+  for (int j = 0; j < kPer; j++) {
+    const int64_t k = base + threadIdx.x + j * kPartThreads;
+    bk[j] = k < n ? bucket(k) : 0xFFFFFFFFu;
   }
+#pragma unroll
+  for (int j = 0; j < kPer; j++)
+    if (bk[j] != 0xFFFFFFFFu) atomicAdd(&h[bk[j]], 1u);
   __syncthreads();
   for (int b = threadIdx.x; b < nbuckets; b += blockDim.x) hist[(int64_t)b * ntiles + blockIdx.x] = h[b];
 }
@@ -253,15 +258,21 @@ __global__ void __launch_bounds__(kPartThreads) k_part_scatter(BucketF bucket, M
   uint32_t rank[kPartItems];
   uint32_t bk[kPartItems];
   uint64_t va[kPartItems], vb[kPartItems];
+  // all loads of the chunk in flight before the first use (the ballots and
+  // __syncwarp below would otherwise serialise one HBM round trip per item)
+#pragma unroll
+  for (int r = 0; r < kPartItems; r++) {
+    const int64_t k = cbase + r * 32 + lane;
+    va[r] = 0;
+    vb[r] = 0;
+    if (k < n) move.load(k, va[r], vb[r]);
+  }
 #pragma unroll
   for (int r = 0; r < kPartItems; r++) {
     int64_t k = cbase + r * 32 + lane;
     bool valid = k < n;
     uint32_t b = 0;
-    if (valid) {
-      b = bucket(k);
-      move.load(k, va[r], vb[r]);
-    }
+    if (valid) b = bucket.of_payload(k, va[r], vb[r]);
     // lanes with the same bucket: one ballot per bucket bit (match.any is
     // slow when a warp holds many distinct values); invalid lanes use 512
     uint32_t peers = kFull;
