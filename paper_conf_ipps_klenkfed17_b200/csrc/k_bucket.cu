@@ -168,6 +168,7 @@ static cudaError_t partition_side(const SnapRead& snap, int64_t n, int nb, uint6
 constexpr int kBucketCap = 1024;   // elements (receives + messages) per bucket on chip
 constexpr int kBucketThreads = 256;
 constexpr uint32_t kBucketH = 2048;  // hash slots (>= 2 * kBucketCap)
+constexpr uint32_t kMaxRun = 64;     // ordered: longest run of one tuple walked on chip
 
 struct BucketArgs {
   FlatArgs a;
@@ -180,32 +181,30 @@ struct BucketArgs {
   uint32_t* overflow;
 };
 
+// Elements of a bucket are kept in snapshot order (the partition is stable),
+// so an element's bucket position orders it among the equal tuples of its
+// side.  Tuples are found through an open-addressing table of 32-bit entries
+// (16-bit fingerprint | representative element); the elements of a tuple form
+// singly linked lists per side, pushed with one atomic exchange each.
 template <bool ORDERED>
 struct BucketSmem {
-  uint64_t hdr[kBucketCap];      // receives [0, nr), then messages [nr, nr + nm)
-  uint32_t idx[kBucketCap];      // snapshot index
-  uint16_t key[kBucketCap];      // tuple id | kNone
-  uint16_t rank[kBucketCap];     // rank among the equal tuples of the element's side
-  uint16_t table[kBucketH];      // slot -> representative message (element index)
-  uint16_t cnt_m[kBucketCap];    // messages per tuple
-  uint16_t start_m[kBucketCap];  // start of the tuple in by_key
-  uint16_t cnt_r[kBucketCap];    // receives per tuple
-  uint16_t by_key[kBucketCap];   // messages grouped by tuple, in rank order (element index)
-  uint16_t pcnt[ORDERED ? 4 : 2][kBucketCap];  // per-half counts / running ranks (msgs, then receives)
-  uint32_t scan[kBucketThreads / 32 + 1];
-  uint32_t K;
-  uint32_t matched;
+  uint64_t hdr[kBucketCap];               // receives [0, nr), then messages [nr, nr + nm)
+  uint32_t idx[kBucketCap];               // snapshot index
+  uint32_t table[kBucketH];               // tuple table
+  uint16_t mhead[kBucketH];               // per slot: message list
+  uint16_t rhead[ORDERED ? kBucketH : 2];  // per slot: receive list (ordered)
+  uint16_t next[kBucketCap];              // list links
+  uint16_t slot[kBucketCap];              // receive -> slot | kNone
+  uint16_t rank[ORDERED ? kBucketCap : 2];  // message rank among its tuple's messages
+  uint32_t matched[kBucketCap / 32];      // message matched bits (by message offset)
 };
 
 template <bool ORDERED>
 __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   BucketSmem<ORDERED>& sm = *reinterpret_cast<BucketSmem<ORDERED>*>(smem_raw);
-  constexpr int QN = ORDERED ? 2 : 1;  // ordered: each side placed in two halves by two warps
-  constexpr int RROW = QN;             // first pcnt row of the receive side
   constexpr int NT = kBucketThreads;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint32_t lt = lanemask_lt();
+  const int tid = threadIdx.x, lane = tid & 31;
   const FlatArgs& a = ba.a;
   const int b = blockIdx.x;
   const uint32_t r0 = ba.roff[b], nr = ba.roff[b + 1] - r0;
@@ -218,152 +217,137 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
   const uint32_t n = nr + nm;
   const int64_t rres = a.R.q_len[0], rpb = a.R.pend_begin(0);
   const int64_t mres = a.M.q_len[0], mpb = a.M.pend_begin(0);
-  const uint32_t hmask = kBucketH - 1;
-  for (uint32_t e = tid; e < n; e += NT) {
-    if (e < nr) {
-      sm.hdr[e] = ba.rh[r0 + e];
-      sm.idx[e] = (uint32_t)ba.ri[r0 + e];
-    } else {
-      sm.hdr[e] = ba.mh[m0 + e - nr];
-      sm.idx[e] = (uint32_t)ba.mi[m0 + e - nr];
+  constexpr uint32_t hmask = kBucketH - 1;
+  // load (all loads of a thread in flight), clear the tables
+  {
+    constexpr int PER = kBucketCap / NT;
+    uint64_t hv[PER], iv[PER];
+#pragma unroll
+    for (int u = 0; u < PER; u++) {
+      const uint32_t e = tid + u * NT;
+      hv[u] = 0;
+      iv[u] = 0;
+      if (e < nr) {
+        hv[u] = ba.rh[r0 + e];
+        iv[u] = ba.ri[r0 + e];
+      } else if (e < n) {
+        hv[u] = ba.mh[m0 + e - nr];
+        iv[u] = ba.mi[m0 + e - nr];
+      }
+    }
+    for (uint32_t s = tid; s < kBucketH / 4; s += NT) reinterpret_cast<uint4*>(sm.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
+    for (uint32_t s = tid; s < kBucketH / 8; s += NT) reinterpret_cast<uint4*>(sm.mhead)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
+    if (ORDERED)
+      for (uint32_t s = tid; s < kBucketH / 8; s += NT) reinterpret_cast<uint4*>(sm.rhead)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
+    for (uint32_t s = tid; s < kBucketCap / 32; s += NT) sm.matched[s] = 0u;
+#pragma unroll
+    for (int u = 0; u < PER; u++) {
+      const uint32_t e = tid + u * NT;
+      if (e < n) {
+        sm.hdr[e] = hv[u];
+        sm.idx[e] = (uint32_t)iv[u];
+      }
     }
   }
-  for (uint32_t s = tid; s < kBucketH / 2; s += NT) reinterpret_cast<uint32_t*>(sm.table)[s] = 0xFFFFFFFFu;
-  if (tid == 0) {
-    sm.matched = 0;
-    sm.K = 0;
-  }
   __syncthreads();
-  // message tuples into the hash table (slot -> representative element); the
-  // CAS winner takes the next dense id and records it in rank[representative]
-  // (rank is only filled later, by the ranking step)
+  // messages: find or open the tuple's slot, push onto its message list
   for (uint32_t e = nr + tid; e < n; e += NT) {
     const uint64_t h = sm.hdr[e];
-    uint32_t s = slot_hash(h) & hmask;
+    const uint64_t p = h * 0xD6E8FEB86659FD93ull;
+    uint32_t s = (uint32_t)(p >> 40) & hmask;
+    const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
     while (true) {
-      uint16_t o = sm.table[s];
-      if (o == kEmpty16) {
-        o = cas16(&sm.table[s], kEmpty16, (uint16_t)e);
-        if (o == kEmpty16) {
-          const uint32_t id = atomicAdd(&sm.K, 1u);
-          sm.rank[e] = (uint16_t)id;
-#pragma unroll
-          for (int q = 0; q < 2 * QN; q++) sm.pcnt[q][id] = 0;
-          o = (uint16_t)e;
-          break;
-        }
+      uint32_t o = sm.table[s];
+      if (o == 0xFFFFFFFFu) {
+        o = atomicCAS(&sm.table[s], 0xFFFFFFFFu, (fp << 16) | e);  // representative's header is in smem already
+        if (o == 0xFFFFFFFFu) break;
       }
-      if (sm.hdr[o] == h) break;
+      if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) break;
       s = (s + 1) & hmask;
     }
-    sm.key[e] = (uint16_t)(s);  // slot for now
+    sm.next[e] = exch16(&sm.mhead[s], (uint16_t)e);
   }
   __syncthreads();
-  const uint32_t K = sm.K;
-  // tuple ids; per-half counts (ordered) or plain counts (unordered)
-  for (uint32_t e = tid; e < n; e += NT) {
-    uint16_t k;
-    const bool is_msg = e >= nr;
-    if (is_msg) {
-      k = sm.rank[sm.table[sm.key[e]]];
-    } else {
+  // receives: look the tuple up (ordered: push onto its receive list)
+  for (uint32_t e = tid; e < nr; e += NT) {
+    const uint64_t h = sm.hdr[e];
+    const uint64_t p = h * 0xD6E8FEB86659FD93ull;
+    uint32_t s = (uint32_t)(p >> 40) & hmask;
+    const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
+    uint32_t found = kNone;
+    while (true) {
+      const uint32_t o = sm.table[s];
+      if (o == 0xFFFFFFFFu) break;
+      if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) {
+        found = s;
+        break;
+      }
+      s = (s + 1) & hmask;
+    }
+    sm.slot[e] = (uint16_t)found;
+    if (ORDERED && found != kNone) sm.next[e] = exch16(&sm.rhead[found], (uint16_t)e);
+  }
+  if (ORDERED) {
+    // message ranks: earlier messages of the same tuple have smaller positions
+    for (uint32_t e = nr + tid; e < n; e += NT) {
       const uint64_t h = sm.hdr[e];
-      uint32_t s = slot_hash(h) & hmask;
-      k = kNone;
+      const uint64_t p = h * 0xD6E8FEB86659FD93ull;
+      uint32_t s = (uint32_t)(p >> 40) & hmask;
+      const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
       while (true) {
-        const uint16_t o = sm.table[s];
-        if (o == kEmpty16) break;
-        if (sm.hdr[o] == h) {
-          k = sm.rank[o];
-          break;
-        }
+        const uint32_t o = sm.table[s];
+        if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) break;
         s = (s + 1) & hmask;
       }
-    }
-    sm.key[e] = k;
-    if (k != kNone) {
-      const uint32_t side_n = is_msg ? nm : nr, x = is_msg ? e - nr : e;
-      const uint32_t q = ORDERED ? (uint32_t)(((uint64_t)x * QN) / side_n) : 0u;
-      inc16(&sm.pcnt[(is_msg ? 0 : RROW) + q][k]);
-    }
-  }
-  __syncthreads();
-  {  // per tuple: quarter prefixes, totals, message list starts
-    const uint32_t per = (K + NT - 1) / NT;
-    const uint32_t k0 = min(K, tid * per), k1 = min(K, k0 + per);
-    uint32_t c = 0;
-    for (uint32_t k = k0; k < k1; k++) {
-      uint32_t rm = 0, rr = 0;
-#pragma unroll
-      for (int q = 0; q < QN; q++) {
-        const uint32_t x = sm.pcnt[q][k], y = sm.pcnt[RROW + q][k];
-        sm.pcnt[q][k] = (uint16_t)rm;
-        sm.pcnt[RROW + q][k] = (uint16_t)rr;
-        rm += x;
-        rr += y;
-      }
-      sm.cnt_m[k] = (uint16_t)rm;
-      sm.cnt_r[k] = (uint16_t)rr;
-      c += rm;
-    }
-    uint32_t tot;
-    uint32_t st = block_excl_scan<uint32_t>(c, sm.scan, &tot);
-    for (uint32_t k = k0; k < k1; k++) {
-      sm.start_m[k] = (uint16_t)st;
-      st += sm.cnt_m[k];
-    }
-  }
-  __syncthreads();
-  // ranks
-  if (ORDERED && warp < 2 * QN) {
-    const bool msg_side = warp < QN;
-    const int q = warp % QN;
-    const uint32_t side_n = msg_side ? nm : nr, base = msg_side ? nr : 0;
-    const int64_t x0 = ((int64_t)side_n * q + QN - 1) / QN, x1 = ((int64_t)side_n * (q + 1) + QN - 1) / QN;
-    place_in_order(
-        x1 - x0, [&](int64_t x) { return (uint32_t)sm.key[base + x0 + x]; }, sm.start_m, sm.pcnt[warp],
-        [&](int64_t x, uint32_t k, uint32_t r, uint32_t slot) {
-          const uint32_t e = base + (uint32_t)(x0 + x);
-          sm.rank[e] = (uint16_t)r;
-          if (msg_side) sm.by_key[slot] = (uint16_t)e;
-        },
-        lane, lt, K);
-  } else if (!ORDERED) {
-    for (uint32_t e = tid; e < n; e += NT) {
-      const uint16_t k = sm.key[e];
-      if (k == kNone) continue;
-      const bool is_msg = e >= nr;
-      const uint32_t r = fetch_inc16(&sm.pcnt[is_msg ? 0 : RROW][k]);
+      uint32_t r = 0, len = 0;
+      for (uint32_t x = sm.mhead[s]; x != kNone && len <= kMaxRun; x = sm.next[x], len++) r += x < e;
+      if (len > kMaxRun) atomicOr(ba.overflow, 1u);  // a tuple too long to rank by walking
       sm.rank[e] = (uint16_t)r;
-      if (is_msg) sm.by_key[sm.start_m[k] + r] = (uint16_t)e;
     }
   }
   __syncthreads();
-  // results in bucket order (coalesced): receive at bucket-sorted position
-  // r0 + e, message flags at m0 + e - nr; the queue compaction reads the same
-  // order, so per-tuple order (all these levels need) is kept
+  // receives take their message: ordered -- the message of equal rank;
+  // unordered -- any message of the tuple (pop from the list)
   uint32_t nmatch = 0;
-  for (uint32_t e = tid; e < n; e += NT) {
-    const uint16_t k = sm.key[e];
-    const uint32_t u = sm.idx[e];
-    if (e < nr) {
-      int64_t mc = MM_NO_MATCH;
-      uint8_t f = 0;
-      if (k != kNone && sm.rank[e] < sm.cnt_m[k]) {
-        const uint32_t j = sm.by_key[sm.start_m[k] + sm.rank[e]];
-        mc = a.M.cookie(0, sm.idx[j], mres, mpb);
-        f = 1;
-        nmatch++;
+  for (uint32_t e = tid; e < nr; e += NT) {
+    const uint32_t s = sm.slot[e];
+    uint32_t j = kNone;
+    if (s != kNone) {
+      if (ORDERED) {
+        uint32_t r = 0, len = 0;
+        for (uint32_t x = sm.rhead[s]; x != kNone && len <= kMaxRun; x = sm.next[x], len++) r += x < e;
+        if (len > kMaxRun) atomicOr(ba.overflow, 1u);
+        for (uint32_t x = sm.mhead[s]; x != kNone; x = sm.next[x])
+          if (sm.rank[x] == r) {
+            j = x;
+            break;
+          }
+      } else {
+        uint32_t hd = sm.mhead[s];
+        while (hd != kNone) {  // pops only in this phase: no ABA
+          const uint32_t got = cas16(&sm.mhead[s], (uint16_t)hd, sm.next[hd]);
+          if (got == hd) {
+            j = hd;
+            break;
+          }
+          hd = got;
+        }
       }
-      a.out_rc[r0 + e] = a.R.cookie(0, u, rres, rpb);
-      a.out_mc[r0 + e] = mc;
-      a.rflag[r0 + e] = f;
-    } else {
-      a.mflag[m0 + e - nr] = (k != kNone && sm.rank[e] < sm.cnt_r[k]) ? 1 : 0;
     }
+    int64_t mc = MM_NO_MATCH;
+    if (j != kNone) {
+      atomicOr(&sm.matched[(j - nr) >> 5], 1u << ((j - nr) & 31));
+      mc = a.M.cookie(0, sm.idx[j], mres, mpb);
+      nmatch++;
+    }
+    a.out_rc[r0 + e] = a.R.cookie(0, sm.idx[e], rres, rpb);
+    a.out_mc[r0 + e] = mc;
+    a.rflag[r0 + e] = j != kNone ? 1 : 0;
   }
   for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
   if (lane == 0 && nmatch) atomicAdd(a.n_matched, (unsigned long long)nmatch);
+  __syncthreads();
+  for (uint32_t x = tid; x < nm; x += NT) a.mflag[m0 + x] = (sm.matched[x >> 5] >> (x & 31)) & 1u;
 }
 
 // ~512 elements per bucket on average (capacity 1024: a bucket overflows

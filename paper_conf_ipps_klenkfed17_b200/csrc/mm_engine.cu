@@ -123,7 +123,8 @@ struct Queue {
   Pending pend;
   int64_t seq = 0;
   int cur = 0;
-  int64_t resid_host = 0;  // exact residual count (single-endpoint levels)
+  int64_t resid_host = 0;  // residual count (single-endpoint levels): exact if resid_exact, else an upper bound
+  bool resid_exact = true;
 };
 
 }  // namespace
@@ -321,7 +322,10 @@ static int materialize(mm_engine* e, Queue& q, int64_t cap) {
   CK(launch_materialize(s, e->n_ep, (uint64_t*)q.hdr[q.cur].p, (int64_t*)q.cookie[q.cur].p, (int32_t*)q.len[q.cur].p,
                         (uint32_t*)e->err.p, e->st));
   q.resid_host += q.pend.n;
-  if (q.resid_host > cap) q.resid_host = cap;
+  if (q.resid_host > cap) {
+    q.resid_host = cap;
+    q.resid_exact = false;
+  }
   q.pend = Pending();
   return MM_OK;
 }
@@ -396,6 +400,7 @@ int mm_reset(mm_engine* e) {
     q->seq = 0;
     q->cur = 0;
     q->resid_host = 0;
+    q->resid_exact = true;
   }
   CK(cudaMemsetAsync(e->err.p, 0, 4, e->st));
   return MM_OK;
@@ -474,10 +479,18 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
   Side R = make_side(e, e->rq, e->rcap), M = make_side(e, e->mq, e->mcap);
   // exact residual sizes (and, for the sort, the varying header bits)
   const int64_t bound = e->rq.resid_host + R.p_n + e->mq.resid_host + M.p_n;
-  CK(launch_snapshot_info(R, M, bound, (SnapInfo*)e->info.p, ordered, e->st));
-  SnapInfo info;
-  CK(cudaMemcpyAsync(&info, e->info.p, sizeof(SnapInfo), cudaMemcpyDeviceToHost, e->st));
-  CK(cudaStreamSynchronize(e->st));
+  // the varying header bits (diff) are only needed by the global sort; the
+  // residual sizes are read back only when the host does not know them
+  bool have_diff = ordered && e->flat_kernel != MM_FLAT_KERNEL_BUCKETED;
+  SnapInfo info{};
+  if (have_diff || !e->rq.resid_exact || !e->mq.resid_exact) {
+    CK(launch_snapshot_info(R, M, bound, (SnapInfo*)e->info.p, have_diff, e->st));
+    CK(cudaMemcpyAsync(&info, e->info.p, sizeof(SnapInfo), cudaMemcpyDeviceToHost, e->st));
+    CK(cudaStreamSynchronize(e->st));
+  } else {
+    info.rres = (int32_t)e->rq.resid_host;
+    info.mres = (int32_t)e->mq.resid_host;
+  }
   const int64_t nr = info.rres + R.p_n, nm = info.mres + M.p_n;
   if (nr > e->rcap || nm > e->mcap) return MM_ERR_CAPACITY;
   if (nr > out_cap) return MM_ERR_CAPACITY;
@@ -525,6 +538,12 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
       CK(cudaMemsetAsync(e->nmatched.p, 0, 8, e->st));
     }
   }
+  if (!done && ordered && !have_diff) {
+    CK(launch_snapshot_info(R, M, bound, (SnapInfo*)e->info.p, true, e->st));
+    CK(cudaMemcpyAsync(&info, e->info.p, sizeof(SnapInfo), cudaMemcpyDeviceToHost, e->st));
+    CK(cudaStreamSynchronize(e->st));
+    have_diff = true;
+  }
   if (!done && ordered) {
     SortScratch s;
     for (int b = 0; b < 2; b++) {
@@ -570,6 +589,7 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
     q.cur = nb;
     q.pend = Pending();
     q.resid_host = ns[i];  // upper bound until the next exact read
+    q.resid_exact = false;
   }
   CK(launch_finalize(nullptr, nr, (const unsigned long long*)e->nmatched.p, (int64_t*)e->counts_dev.p, e->st));
   if (counts && !counts_host) CK(cudaMemcpyAsync(counts, e->counts_dev.p, 16, cudaMemcpyDeviceToDevice, e->st));
@@ -627,6 +647,7 @@ int mm_query(mm_engine* e, int64_t* vals) {
   if (e->sem != MM_SEM_MPI) {
     e->rq.resid_host = rsum;
     e->mq.resid_host = msum;
+    e->rq.resid_exact = e->mq.resid_exact = true;
   }
   return err ? MM_ERR_CAPACITY : MM_OK;
 }

@@ -38,6 +38,19 @@ __device__ __forceinline__ uint16_t cas16(uint16_t* p, uint16_t expect, uint16_t
   }
 }
 
+// 16-bit exchange through the containing 32-bit word.
+__device__ __forceinline__ uint16_t exch16(uint16_t* p, uint16_t v) {
+  uint32_t* w = word_of(p);
+  const uint32_t sh = (reinterpret_cast<uintptr_t>(p) & 2) ? 16u : 0u;
+  uint32_t old = *w;
+  while (true) {
+    const uint32_t nw = (old & ~(0xFFFFu << sh)) | ((uint32_t)v << sh);
+    const uint32_t got = atomicCAS(w, old, nw);
+    if (got == old) return (uint16_t)(old >> sh);
+    old = got;
+  }
+}
+
 // 16-bit counter increment through the containing 32-bit word (no carry out:
 // counts stay below 65536).
 __device__ __forceinline__ void inc16(uint16_t* p) {
