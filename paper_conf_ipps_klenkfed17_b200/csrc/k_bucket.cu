@@ -39,9 +39,11 @@ __device__ __forceinline__ uint32_t bucket_of(uint64_t h, int nb) {
 
 
 struct SnapRead {
-  Side S;
-  int64_t resid, pb;
-  __device__ __forceinline__ uint64_t hdr(int64_t u) const { return S.hdr(0, u, resid, pb); }
+  // snapshot element u: residual queue entries [0, resid), then the pending batch
+  const uint64_t* q;  // residual headers (endpoint 0)
+  const uint64_t* p;  // pending headers (nullptr if none)
+  int64_t resid;
+  __device__ __forceinline__ uint64_t hdr(int64_t u) const { return u < resid ? q[u] : p[u - resid]; }
 };
 
 // payload of a partitioned element: header word + (bucket << 32 | snapshot index)
@@ -361,11 +363,8 @@ int64_t bucket_bits_for(int64_t n) {
 cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cudaStream_t st) {
   const int nb = (int)bucket_bits_for(a.nr + a.nm);
   const uint32_t B = 1u << nb;
-  SnapRead rs{a.R, 0, 0}, ms{a.M, 0, 0};
-  rs.resid = s.rres;
-  ms.resid = s.mres;
-  rs.pb = 0;  // single endpoint: pending batch starts at 0
-  ms.pb = 0;
+  // single endpoint: the pending batch starts at 0
+  SnapRead rs{a.R.q_hdr, a.R.p_hdr, s.rres}, ms{a.M.q_hdr, a.M.p_hdr, s.mres};
   uint64_t *rh, *mh;
   uint64_t *ri, *mi;
   cudaError_t err = partition_side(rs, a.nr, nb, s.h[0], s.i[0], s.h[1], s.i[1], s.part, s.roff, &rh, &ri, st);

@@ -204,8 +204,8 @@ constexpr int kPartWarps = 8;
 constexpr int kPartThreads = kPartWarps * 32;
 constexpr int kPartItems = 8;                           // per lane
 constexpr int kPartMaxBuckets = 512;
-constexpr int kPartWarpChunk = 32 * kPartItems;         // 512
-constexpr int kPartTile = kPartWarps * kPartWarpChunk;  // 4096
+constexpr int kPartWarpChunk = 32 * kPartItems;         // 256 elements per warp
+constexpr int kPartTile = kPartWarps * kPartWarpChunk;  // 2048 elements per tile
 
 // hist[b * ntiles + tile] = elements of tile with bucket b.
 template <class BucketF>
@@ -215,7 +215,7 @@ __global__ void __launch_bounds__(kPartThreads) k_part_hist(BucketF bucket, int6
   for (int b = threadIdx.x; b < kPartMaxBuckets; b += blockDim.x) h[b] = 0;
   __syncthreads();
   const int64_t base = (int64_t)blockIdx.x * kPartTile;
-  constexpr int kPer = kPartTile / kPartThreads;  // 16 elements per thread, all loads in flight
+  constexpr int kPer = kPartTile / kPartThreads;  // elements per thread, all loads in flight
   uint32_t bk[kPer];
 #pragma unroll
   for (int j = 0; j < kPer; j++) {
