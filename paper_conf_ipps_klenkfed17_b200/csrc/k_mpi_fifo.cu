@@ -371,6 +371,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       continue;  // uniform across the CTA
     }
     const uint32_t nr = (uint32_t)nr64, nm = (uint32_t)nm64;
+    const EpSide RS(a.R, e, rres, rpb), MS(a.M, e, mres, mpb);
     // quarter boundaries: element x is in quarter q iff qb[q] <= x < qb[q + 1]
     const uint32_t mq1 = (nm + 3) / 4, mq2 = (2 * nm + 3) / 4, mq3 = (3 * nm + 3) / 4;
     const uint32_t rq1 = (nr + 3) / 4, rq2 = (2 * nr + 3) / 4, rq3 = (3 * nr + 3) / 4;
@@ -398,7 +399,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
 #pragma unroll
       for (int u = 0; u < 4; u++) {  // read once from HBM, four loads in flight
         const uint32_t j = j0 + u * NT;
-        hv[u] = j < nm ? a.M.hdr(e, j, mres, mpb) : 0ull;
+        hv[u] = j < nm ? MS.hdr(j) : 0ull;
       }
 #pragma unroll
       for (int u = 0; u < 4; u++) {
@@ -448,7 +449,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
 #pragma unroll
       for (int u = 0; u < 4; u++) {  // four independent HBM loads in flight
         const uint32_t i = i0 + u * NT;
-        hv[u] = i < nr ? a.R.hdr(e, i, rres, rpb) : 0ull;
+        hv[u] = i < nr ? RS.hdr(i) : 0ull;
       }
 #pragma unroll
       for (int u = 0; u < 4; u++) {
@@ -528,7 +529,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       uint32_t wp = (uint32_t)(ex >> 32);
       for (uint32_t i = i0; i < i1 && wc; i++)
         if (ws.recv_key[i] == kWild) {
-          if (wp < L.wcap) ws.whdr[wp] = a.R.hdr(e, i, rres, rpb);
+          if (wp < L.wcap) ws.whdr[wp] = RS.hdr(i);
           ws.recv_e[i] = (uint16_t)wp;
           ws.wl[wp++] = (uint16_t)i;
         }
@@ -537,7 +538,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     __syncthreads();
     // header of the x-th wildcard (staged for the first wcap of them)
     auto hdrof = [&](uint32_t x) -> uint64_t {
-      return x < L.wcap ? ws.whdr[x] : a.R.hdr(e, ws.wl[x], rres, rpb);
+      return x < L.wcap ? ws.whdr[x] : RS.hdr(ws.wl[x]);
     };
     MM_PHASE(5);
     // P6 -------------------------------------------------------------------
@@ -729,7 +730,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           rcv[u] = 0;
           if (i < nr) {
             uint32_t res = kNone;
-            const int64_t rc = a.R.cookie(e, i, rres, rpb);
+            const int64_t rc = RS.cookie(i);
             const uint16_t rk = ws.recv_key[i];
             if (rk == kWild) {
               res = ws.recv_res[ws.recv_e[i]];
@@ -743,12 +744,12 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             a.out_rc[obase + i] = rc;
             if (res != kNone) {
               atomicOr(&ws.matched[res >> 5], 1u << (res & 31));
-              a.out_mc[obase + i] = a.M.cookie(e, res, mres, mpb);
+              a.out_mc[obase + i] = MS.cookie(res);
               nmatch++;
             } else {
               a.out_mc[obase + i] = (int64_t)MM_NO_MATCH;
               fld |= 1ull << (16 * u);
-              rh[u] = a.R.hdr(e, i, rres, rpb);
+              rh[u] = RS.hdr(i);
               rcv[u] = rc;
             }
           }
@@ -786,8 +787,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           mc[u] = 0;
           if (j < nm && !((ws.matched[j >> 5] >> (j & 31)) & 1u)) {
             fld |= 1ull << (16 * u);
-            mh[u] = a.M.hdr(e, j, mres, mpb);
-            mc[u] = a.M.cookie(e, j, mres, mpb);
+            mh[u] = MS.hdr(j);
+            mc[u] = MS.cookie(j);
           }
         }
         uint64_t tot;

@@ -85,6 +85,31 @@ struct Side {
   }
 };
 
+// One endpoint's snapshot side with the per-endpoint address arithmetic done
+// once: element k < resid is queue entry k, element k >= resid pending entry
+// k - resid (the pending pointers are pre-offset by -resid).
+struct EpSide {
+  const uint64_t* qh;
+  const int64_t* qc;
+  const uint64_t* ph;
+  const int64_t* pc;
+  int64_t cseq;  // computed cookie of pending element k: cseq + k
+  uint32_t resid;
+  __device__ __forceinline__ EpSide(const Side& S, int e, int64_t res, int64_t pb) {
+    qh = S.q_hdr + (int64_t)e * S.cap;
+    qc = S.q_cookie + (int64_t)e * S.cap;
+    ph = S.p_hdr ? S.p_hdr + (pb - res) : nullptr;
+    pc = S.p_cookie ? S.p_cookie + (pb - res) : nullptr;
+    cseq = S.p_seq0 + pb - res;
+    resid = (uint32_t)res;
+  }
+  __device__ __forceinline__ uint64_t hdr(uint32_t k) const { return k < resid ? qh[k] : ph[k]; }
+  __device__ __forceinline__ int64_t cookie(uint32_t k) const {
+    if (k < resid) return qc[k];
+    return pc ? pc[k] : cseq + (int64_t)k;
+  }
+};
+
 // ------------------------------------------------------------ block scans
 template <class T>
 __device__ __forceinline__ T warp_incl_scan(T v) {
