@@ -206,92 +206,6 @@ __device__ __forceinline__ void resolve_wildcard(const FifoWs& ws, uint32_t x, u
   __syncwarp();
 }
 
-// A chain of wildcard receives over at most 32 candidate tuples, one tuple per
-// lane (own, k) with its cursor and claim count in registers.  gen(x, w, r)
-// yields the wildcards in posting order (x = index into wl, w = posting
-// position, r = header when test_admit) and false at the end; it is
-// warp-uniform and serves positions from registers (a chunk of 32 loaded at a
-// time).  The head a lane offers at step t is list_k[e_k(w_t) + c]; e_k(w_t)
-// does not depend on the chain (the cursor keeps the position of the next
-// exact receive of k in a register, so it usually moves without a load) and c
-// grows by one only when the lane wins, so the window list_k[e + c .. e + c + 3]
-// of the NEXT step is formed (mostly from registers) while the current step
-// resolves: the critical path of a wildcard is one redux.sync.min and a
-// select.
-// test_admit: wildcards may differ, so each lane tests admission with the
-// masked XOR; otherwise every wildcard admits every candidate (a group).
-template <class GenF>
-__device__ __forceinline__ void register_chain(const FifoWs& ws, bool own, uint32_t k, GenF gen, bool test_admit,
-                                               int lane) {
-  uint32_t x, w;
-  uint64_t r;
-  if (!gen(x, w, r)) return;
-  uint32_t cur = 0, c = 0, rs = 0, rc = 0, st = 0, cnt = 0, npos = 0xFFFFFFFFu;
-  uint64_t kh = 0;
-  if (own) {
-    rs = ws.key_rstart[k];
-    rc = ws.key_rcnt[k];
-    st = ws.key_start[k];
-    cnt = ws.key_cnt[k];
-    kh = ws.keyhdr[k];
-    if (rc) npos = ws.rby_key[rs];
-  }
-  auto head_at = [&](uint32_t i) { return (own && i < cnt) ? (uint32_t)ws.by_key[st + i] : 0xFFFFFFFFu; };
-  // cursor: exact receives of k posted before w (monotone in w); npos = the
-  // posting position of the next one
-  auto advance = [&](uint32_t w) {
-    while (npos < w) {
-      cur++;
-      npos = cur < rc ? (uint32_t)ws.rby_key[rs + cur] : 0xFFFFFFFFu;
-    }
-  };
-  advance(w);
-  uint32_t h0 = head_at(cur + c), h1 = head_at(cur + c + 1), h2 = head_at(cur + c + 2);
-  while (true) {
-    // the next step's window, independent of this step's outcome
-    uint32_t xn, wn;
-    uint64_t rn;
-    const bool more = gen(xn, wn, rn);
-    uint32_t y0 = h0, y1 = h1, y2 = h2, y3 = 0xFFFFFFFFu;
-    if (more) {
-      const uint32_t cur0 = cur;
-      advance(wn);
-      const uint32_t d = cur - cur0, b = cur + c;
-      if (d == 0) {
-        y3 = head_at(b + 3);
-      } else if (d == 1) {
-        y0 = h1;
-        y1 = h2;
-        y2 = head_at(b + 2);
-        y3 = head_at(b + 3);
-      } else {
-        y0 = head_at(b);
-        y1 = head_at(b + 1);
-        y2 = head_at(b + 2);
-        y3 = head_at(b + 3);
-      }
-    }
-    uint32_t cand = h0;
-    if (test_admit && ((kh ^ r) & wildcard_mask(r)) != 0) cand = 0xFFFFFFFFu;
-    const uint32_t win = __reduce_min_sync(kFull, cand);
-    const bool won = win != 0xFFFFFFFFu && cand == win;
-    if (won) {
-      ws.wlog[st + c] = (uint16_t)w;
-      c++;
-    }
-    if (lane == 0) ws.recv_res[x] = win == 0xFFFFFFFFu ? kNone : (uint16_t)win;
-    if (!more) break;
-    // next step's heads: list_k[cur' + c'] with c' = c (+1 if won)
-    h0 = won ? y1 : y0;
-    h1 = won ? y2 : y1;
-    h2 = won ? y3 : y2;
-    x = xn;
-    w = wn;
-    r = rn;
-  }
-  if (own) ws.key_c[k] = (uint16_t)c;
-}
-
 // Wildcard chain by a walk over the receive queue in posting order, 32
 // receives at a time (used when all tuples fit in one warp, K <= 32).  Lane l
 // owns tuple l.  Per chunk each exact receive sets bit j (its chunk offset) in
@@ -343,6 +257,69 @@ __device__ __forceinline__ void stream_chain(const FifoWs& ws, uint32_t* kmask, 
     __syncwarp();
   }
   if (own) ws.key_c[lane] = (uint16_t)c;
+}
+
+// The wildcard chain in its leanest form (about twenty instructions a step).
+// Lane l owns tuple k (own) and keeps, in registers, its next exact receive's
+// posting position (npos) and a window h0/h1 = list_k[cur + c], list_k[cur +
+// c + 1] of its message list: an exact receive of k posted before the
+// wildcard (cur++) and a win (c++) both shift the window by one.  Wildcards
+// are served in posting order from wl[x_begin..W) -- those with in(y) --, 32
+// positions at a time held in registers; `left` of them in all.  A step is a
+// shuffle, the cursor compare, one redux.sync.min and, for the winner, a
+// store and the window shift.  ADMIT: wildcards may differ in type, so each
+// lane tests admission with the masked XOR.
+template <bool ADMIT, class InF, class HdrF>
+__device__ __forceinline__ void lean_chain(const FifoWs& ws, bool own, uint32_t k, uint32_t x_begin, uint32_t W,
+                                           uint32_t left, InF in_chain, HdrF hdrof, int lane) {
+  uint32_t st = 0, hend = 0, rs = 0, rc = 0;
+  uint64_t kh = 0;
+  if (own) {
+    st = ws.key_start[k];
+    hend = st + ws.key_cnt[k];
+    rs = ws.key_rstart[k];
+    rc = ws.key_rcnt[k];
+    if (ADMIT) kh = ws.keyhdr[k];
+  }
+  uint32_t cur = 0, c = 0, hp = st;
+  uint32_t npos = rc ? (uint32_t)ws.rby_key[rs] : 0xFFFFFFFFu;
+  uint32_t h0 = hp < hend ? (uint32_t)ws.by_key[hp] : 0xFFFFFFFFu;
+  uint32_t h1 = hp + 1 < hend ? (uint32_t)ws.by_key[hp + 1] : 0xFFFFFFFFu;
+  for (uint32_t cb = x_begin & ~31u; left > 0; cb += 32) {
+    const uint32_t y = cb + lane;
+    const bool in = y >= x_begin && y < W && in_chain(y);
+    uint32_t cm = __ballot_sync(kFull, in);
+    const uint32_t wv = in ? (uint32_t)ws.wl[y] : 0u;
+    const uint64_t rv = (ADMIT && in) ? hdrof(y) : 0ull;
+    while (cm) {
+      const int bit = __ffs(cm) - 1;
+      cm &= cm - 1;
+      left--;
+      const uint32_t w = __shfl_sync(kFull, wv, bit);
+      while (npos < w) {  // exact receives of k posted before w take heads first
+        cur++;
+        npos = cur < rc ? (uint32_t)ws.rby_key[rs + cur] : 0xFFFFFFFFu;
+        hp++;
+        h0 = h1;
+        h1 = hp + 1 < hend ? (uint32_t)ws.by_key[hp + 1] : 0xFFFFFFFFu;
+      }
+      uint32_t cand = h0;
+      if (ADMIT) {
+        const uint64_t r = __shfl_sync(kFull, rv, bit);
+        if (((kh ^ r) & wildcard_mask(r)) != 0) cand = 0xFFFFFFFFu;
+      }
+      const uint32_t win = __reduce_min_sync(kFull, cand);
+      if (win != 0xFFFFFFFFu && cand == win) {
+        ws.wlog[st + c] = (uint16_t)w;
+        c++;
+        hp++;
+        h0 = h1;
+        h1 = hp + 1 < hend ? (uint32_t)ws.by_key[hp + 1] : 0xFFFFFFFFu;
+      }
+      if (lane == 0) ws.recv_res[cb + bit] = win == 0xFFFFFFFFu ? kNone : (uint16_t)win;
+    }
+  }
+  if (own) ws.key_c[k] = (uint16_t)c;
 }
 
 template <int NT, bool SMEM>
@@ -639,13 +616,49 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           }
         }
         __syncthreads();
+        // A group with ONE wildcard and few tuples needs no chain: its
+        // wildcard takes the earliest head list_k[e_k(w)] over the group's
+        // tuples (no earlier claims).  One thread per such group, all groups
+        // at once; the warps below serve the rest.
+        for (uint32_t x = tid; x < W; x += NT) {
+          const uint32_t g = ws.w_grp[x];
+          if (g == kNone || ws.gwc[g] != 1) continue;
+          uint32_t kn = 0;
+          for (uint32_t node = g; node != kNone32 && kn <= 8; node = ws.gnext[node]) kn++;
+          if (kn > 8) continue;
+          const uint32_t w = ws.wl[x];
+          uint32_t best = 0xFFFFFFFFu, bestk = 0;
+          for (uint32_t node = g; node != kNone32; node = ws.gnext[node]) {
+            const uint32_t rs = ws.key_rstart[node];
+            uint32_t lo = 0, hi = ws.key_rcnt[node];
+            while (lo < hi) {  // exact receives of the tuple posted before w
+              const uint32_t mid = (lo + hi) >> 1;
+              if (ws.rby_key[rs + mid] < w) lo = mid + 1;
+              else hi = mid;
+            }
+            if (lo < ws.key_cnt[node]) {
+              const uint32_t j = ws.by_key[ws.key_start[node] + lo];
+              if (j < best) {
+                best = j;
+                bestk = node;
+              }
+            }
+          }
+          ws.recv_res[x] = best == 0xFFFFFFFFu ? kNone : (uint16_t)best;
+          if (best != 0xFFFFFFFFu) {
+            ws.wlog[ws.key_start[bestk]] = (uint16_t)w;
+            ws.key_c[bestk] = 1;
+          }
+          ws.gwc[g] = 0;  // served
+        }
+        __syncthreads();
         MM_PHASE(10);
         // warp v serves the groups whose first wildcard it finds with g % NW == v
         const uint32_t v = (uint32_t)(NW - 1 - warp);
         for (uint32_t b = 0; b < W; b += 32) {
           const uint32_t x = b + lane;
           const uint32_t g = x < W ? ws.w_grp[x] : kNone;
-          const bool lead = g != kNone && g % NW == v && ws.gfirst[g] == x;
+          const bool lead = g != kNone && g % NW == v && ws.gfirst[g] == x && ws.gwc[g] != 0;
           uint32_t leaders = __ballot_sync(kFull, lead);
           while (leaders) {
             const int l = __ffs(leaders) - 1;
@@ -662,35 +675,17 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
               node = ws.gnext[node];
             }
             // the group's wildcards in posting order, from its first one
-            uint32_t left = ws.gwc[gg];
-            uint32_t cb = b, cm = __ballot_sync(kFull, g == gg) & (~0u << l);
-            uint32_t wv = g == gg ? ws.wl[x] : 0u;
-            auto gen = [&](uint32_t& xo, uint32_t& wo, uint64_t& ro) -> bool {
-              if (left == 0) return false;
-              while (cm == 0) {  // next chunk holding wildcards of the group
-                cb += 32;
-                const uint32_t y = cb + lane;
-                const bool in = y < W && ws.w_grp[y] == gg;
-                cm = __ballot_sync(kFull, in);
-                wv = in ? ws.wl[y] : 0u;
-              }
-              const int bit = __ffs(cm) - 1;
-              cm &= cm - 1;
-              left--;
-              xo = cb + bit;
-              wo = __shfl_sync(kFull, wv, bit);
-              ro = 0;
-              return true;
-            };
+            const uint32_t left = ws.gwc[gg];
+            const uint32_t x0 = b + l;
+            auto in_group = [&](uint32_t y) { return ws.w_grp[y] == gg; };
             if (kn <= 32) {
-              register_chain(ws, lane < (int)kn, mine, gen, false, lane);
+              lean_chain<false>(ws, lane < (int)kn, mine, x0, W, left, in_group, hdrof, lane);
             } else {  // a group of more than 32 tuples: scan every tuple, admission tested
-              uint32_t xx, ww;
-              uint64_t rr;
-              while (gen(xx, ww, rr)) {
-                const uint64_t r = hdrof(xx);
-                resolve_wildcard(ws, xx, ww, r, wildcard_mask(r), K, [](uint32_t c0) { return c0; }, lane);
-              }
+              for (uint32_t xx = x0; xx < W; xx++)
+                if (ws.w_grp[xx] == gg) {
+                  const uint64_t r = hdrof(xx);
+                  resolve_wildcard(ws, xx, ws.wl[xx], r, wildcard_mask(r), K, [](uint32_t c0) { return c0; }, lane);
+                }
             }
           }
         }
