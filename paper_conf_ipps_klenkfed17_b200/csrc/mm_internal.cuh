@@ -298,8 +298,9 @@ __global__ void __launch_bounds__(kPartThreads) k_part_scatter(BucketF bucket, M
     bool valid = k < n;
     uint32_t b = 0;
     if (valid) b = bucket.of_payload(k, va[r], vb[r]);
-    // lanes with the same bucket: one ballot per bucket bit (match.any is
-    // slow when a warp holds many distinct values); invalid lanes use 512
+    // lanes with the same bucket: one ballot per bucket bit (here, with ten
+    // bits and eight items in flight, cheaper than match.any); invalid lanes
+    // use 512
     uint32_t peers = kFull;
     {
       const uint32_t v = valid ? b : (uint32_t)kPartMaxBuckets;

@@ -63,18 +63,10 @@ __device__ __forceinline__ uint32_t fetch_inc16(uint16_t* p) {
   return hi ? (old >> 16) : (old & 0xFFFFu);
 }
 
-// Lanes holding the same value as this lane, from one ballot per value bit
-// (nbits covers every value in play).  Replaces match.any, whose cost grows
-// with the number of distinct values in the warp.
-__device__ __forceinline__ uint32_t peers_of(uint32_t v, int nbits) {
-  uint32_t m = kFull;
-  for (int b = 0; b < nbits; b++) {
-    const bool bit = (v >> b) & 1u;
-    const uint32_t bb = __ballot_sync(kFull, bit);
-    m &= bit ? bb : ~bb;
-  }
-  return m;
-}
+// Lanes holding the same value as this lane: one match.any.sync (measured on
+// B200 at a constant ~200 cycles of latency whatever the number of distinct
+// values, 2-3x cheaper than one ballot per value bit; tools/micro/peers.cu).
+__device__ __forceinline__ uint32_t peers_of(uint32_t v) { return __match_any_sync(kFull, v); }
 
 // Ordered placement by one warp: element x (0..n) with tuple id key(x) (>=
 // kWild = skip) gets slot start[k] + running[k]; put(x, k, rank, slot).
@@ -82,12 +74,11 @@ __device__ __forceinline__ uint32_t peers_of(uint32_t v, int nbits) {
 template <class KeyF, class PutF>
 __device__ __forceinline__ void place_in_order(int64_t n, KeyF key, const uint16_t* start, uint16_t* running, PutF put,
                                                int lane, uint32_t lt, uint32_t nkeys) {
-  const int nbits = 32 - __clz(nkeys | 1u);  // ids 0..nkeys (nkeys = "skip")
   for (int64_t b = 0; b < n; b += 32) {
     const int64_t x = b + lane;
     const uint32_t k = x < n ? key(x) : 0xFFFFFFFFu;
     const bool ok = k < kWild;
-    const uint32_t peers = peers_of(ok ? k : nkeys, nbits);
+    const uint32_t peers = peers_of(ok ? k : nkeys);  // nkeys = "skip"
     uint32_t run = 0;
     if (ok) run = running[k];
     __syncwarp();
