@@ -121,8 +121,14 @@ int mm_create(mm_engine **out, int32_t semantics, int32_t n_endpoints,
  *   n           number of elements (>= 0).
  * Device buffers are used in place and must stay valid and unchanged until
  * the next mm_match_batch has executed (stream order).  Host buffers are
- * copied inside the call.  A second post (push) before mm_match_batch moves
- * the pending batch into the queues first.
+ * copied by the engine asynchronously (fully so from page-locked memory) and
+ * must stay valid and unchanged until the next mm_match_batch (or
+ * mm_reset) returns.  At the MPI level with host hdr AND host ep_offsets the
+ * copy is deferred to mm_match_batch and issued in endpoint ranges on an
+ * internal copy stream (MM_OPT_PIPELINE_CHUNKS), both queues' range k before
+ * range k + 1, so that it overlaps the matching of earlier ranges.  A second
+ * post (push) before mm_match_batch moves the pending batch into the queues
+ * first.
  */
 int mm_post_recvs(mm_engine *e, const uint64_t *hdr, const int64_t *cookie,
                   const int64_t *ep_offsets, int64_t n);
@@ -150,7 +156,9 @@ int mm_push_msgs(mm_engine *e, const uint64_t *hdr, const int64_t *cookie,
  * receive of a tuple takes the n-th message of that tuple; NOWILD_UNORDERED --
  * a maximal pairing of equal tuples.  Results for MPI and NOWILD_ORDERED are
  * deterministic and bit-identical to the CPU oracle.
- * With host output pointers (or host counts) the call synchronises the stream.
+ * With host output pointers (or host counts) the call synchronises the stream;
+ * at the MPI level host outputs are copied back per endpoint range as soon as
+ * that range is matched (overlapping the next range's copy-in and matching).
  */
 int mm_match_batch(mm_engine *e, int64_t *out_recv_cookie, int64_t *out_msg_cookie,
                    int64_t out_capacity, int64_t *counts);
@@ -201,7 +209,7 @@ int mm_route(const uint64_t *a, const int64_t *b, int64_t n, int32_t world, int3
  *   Both produce identical results.  Returns MM_ERR_ARG for unknown options
  *   or values.
  */
-enum { MM_OPT_MPI_KERNEL = 1, MM_OPT_FLAT_KERNEL = 2 };
+enum { MM_OPT_MPI_KERNEL = 1, MM_OPT_FLAT_KERNEL = 2, MM_OPT_PIPELINE_CHUNKS = 3 };
 enum { MM_MPI_KERNEL_AUTO = 0, MM_MPI_KERNEL_MATRIX = 1, MM_MPI_KERNEL_FIFO = 2 };
 /*   MM_OPT_FLAT_KERNEL: how the no-wildcard levels run --
  *     MM_FLAT_KERNEL_BUCKETED (default): hash-bucketed, one CTA per bucket in
@@ -210,6 +218,10 @@ enum { MM_MPI_KERNEL_AUTO = 0, MM_MPI_KERNEL_MATRIX = 1, MM_MPI_KERNEL_FIFO = 2 
  *     MM_FLAT_KERNEL_GLOBAL: always the global kernels (LSD radix sort-and-rank
  *       for NOWILD_ORDERED, HBM hash table for NOWILD_UNORDERED). */
 enum { MM_FLAT_KERNEL_BUCKETED = 0, MM_FLAT_KERNEL_GLOBAL = 1 };
+/*   MM_OPT_PIPELINE_CHUNKS: endpoint ranges of the MPI level's host-buffer
+ *     pipeline (H2D of range k+1, matching of range k and D2H of range k-1
+ *     overlap on three streams): 0 = auto (4 at >= 256 endpoints, else 1), 1 = off, 2..32 = that many ranges.  Results are identical
+ *     for every value; a change applies to the next post. */
 int mm_set_option(mm_engine *e, int32_t option, int64_t value);
 
 /* mm_strerror -- static description of an MM_* code. */

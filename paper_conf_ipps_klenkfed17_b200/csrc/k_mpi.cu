@@ -72,7 +72,7 @@ __global__ void k_mpi_matrix(MpiArgs a) {
   const int lane = threadIdx.x & 31;
   const int wpb = blockDim.x >> 5;
   const int w = threadIdx.x >> 5;
-  const int e = blockIdx.x * wpb + w;
+  const int e = a.ep0 + blockIdx.x * wpb + w;
   if (e >= a.n_ep) return;  // warp-uniform; no block-wide barriers below
 
   uint64_t* sm_m = smem + (size_t)w * a.warp_smem_words;
@@ -177,7 +177,7 @@ __global__ void k_mpi_matrix(MpiArgs a) {
 }
 
 cudaError_t launch_mpi_matrix(const MpiArgs& a, cudaStream_t st) {
-  if (a.n_ep <= 0) return cudaSuccess;
+  if (a.n_ep <= a.ep0) return cudaSuccess;
   const size_t per_warp = (size_t)a.warp_smem_words * 8;
   int wpb = (int)(96 * 1024 / per_warp);
   if (wpb > 8) wpb = 8;
@@ -185,7 +185,7 @@ cudaError_t launch_mpi_matrix(const MpiArgs& a, cudaStream_t st) {
   const size_t smem = per_warp * wpb;
   cudaError_t err = cudaFuncSetAttribute(k_mpi_matrix, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
-  const int grid = (a.n_ep + wpb - 1) / wpb;
+  const int grid = (a.n_ep - a.ep0 + wpb - 1) / wpb;
   count_launch();
   k_mpi_matrix<<<grid, wpb * 32, smem, st>>>(a);
   return cudaGetLastError();

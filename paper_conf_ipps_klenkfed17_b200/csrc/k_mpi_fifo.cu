@@ -338,7 +338,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
 #ifdef MM_PHASE_TIMING
   long long t_phase = clock64();
 #endif
-  for (int e = blockIdx.x; e < a.n_ep; e += gridDim.x) {
+  for (int e = a.ep0 + blockIdx.x; e < a.n_ep; e += gridDim.x) {
     const int64_t rres = a.R.q_len[e], mres = a.M.q_len[e];
     const int64_t rpb = a.R.pend_begin(e), mpb = a.M.pend_begin(e);
     const int64_t nr64 = rres + a.R.pend_count(e), nm64 = mres + a.M.pend_count(e);
@@ -879,8 +879,8 @@ extern "C" int mm_debug_phase_cycles(unsigned long long* out, int reset) {
 #endif
 
 cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws, cudaStream_t st) {
-  if (a.n_ep <= 0) return cudaSuccess;
-  const int grid = fifo_grid(L, a.n_ep);
+  if (a.n_ep <= a.ep0) return cudaSuccess;
+  const int grid = fifo_grid(L, a.n_ep - a.ep0);
   cudaError_t err;
   if (L.in_smem) {
     err = cudaFuncSetAttribute(k_mpi_fifo<256, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);

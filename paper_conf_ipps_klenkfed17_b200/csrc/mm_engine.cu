@@ -115,12 +115,21 @@ struct Pending {
   int64_t n = 0;
   int64_t seq0 = 0;
   bool active = false;
+  int chunks = 0;  // > 0: host input staged in `chunks` endpoint ranges on the copy stream (Queue::ev)
+  bool issued = false;  // the chunk copies are submitted (deferred so both queues' chunks interleave)
+  const uint64_t* h_hdr = nullptr;  // the caller's host buffers (valid until mm_match_batch returns)
+  const int64_t* h_cookie = nullptr;
+  const int64_t* h_off = nullptr;
 };
+
+// Host-buffer pipeline (MPI level): endpoint range k of C is [k*n_ep/C, (k+1)*n_ep/C).
+constexpr int kMaxChunks = 32;
 
 struct Queue {
   DBuf hdr[2], cookie[2], len[2];  // ping-pong (the MPI level compacts in place and uses [0] only)
   DBuf st_hdr, st_cookie, st_off;   // staging for host inputs
   Pending pend;
+  cudaEvent_t ev[kMaxChunks] = {};  // chunk k of the pending host input is on the device
   int64_t seq = 0;
   int cur = 0;
   int64_t resid_host = 0;  // residual count (single-endpoint levels): exact if resid_exact, else an upper bound
@@ -153,7 +162,22 @@ struct mm_engine {
   long long bucket_fallbacks = 0;
   Timer timer;
   long long launches = 0;
+  // host-buffer pipeline: H2D copies on cs, D2H copies on ds, chunk kernels on st
+  cudaStream_t cs = nullptr, ds = nullptr;
+  cudaEvent_t ev_st = nullptr, ev_k[kMaxChunks] = {};
+  int64_t* h_off = nullptr;  // pinned copy of out_off (n_ep + 1)
+  int pipeline = 0;          // MM_OPT_PIPELINE_CHUNKS (0 = auto)
 };
+
+static int64_t chunk_ep(const mm_engine* e, int k, int C) { return (int64_t)k * e->n_ep / C; }
+
+// Number of endpoint ranges the host-buffer pipeline uses (1 = no pipeline).
+static int pipeline_chunks(const mm_engine* e) {
+  if (e->sem != MM_SEM_MPI || e->n_ep < 2) return 1;
+  int C = e->pipeline;
+  if (C == 0) C = e->n_ep >= 256 ? 4 : 1;
+  return C < e->n_ep ? C : e->n_ep;
+}
 
 // Attributes the library's kernel launches during one API call to an engine.
 struct LaunchScope {
@@ -216,8 +240,19 @@ const char* mm_version(void) { return "mm 0.1.0 sm_100a"; }
 int mm_destroy(mm_engine* e) {
   if (!e) return MM_OK;
   cudaStreamSynchronize(e->st);
+  if (e->cs) cudaStreamSynchronize(e->cs);
+  if (e->ds) cudaStreamSynchronize(e->ds);
   e->timer.destroy();
   Queue* qs[2] = {&e->rq, &e->mq};
+  for (int k = 0; k < kMaxChunks; k++) {
+    if (e->ev_k[k]) cudaEventDestroy(e->ev_k[k]);
+    for (Queue* q : qs)
+      if (q->ev[k]) cudaEventDestroy(q->ev[k]);
+  }
+  if (e->ev_st) cudaEventDestroy(e->ev_st);
+  if (e->cs) cudaStreamDestroy(e->cs);
+  if (e->ds) cudaStreamDestroy(e->ds);
+  if (e->h_off) cudaFreeHost(e->h_off);
   for (Queue* q : qs) {
     for (int b = 0; b < 2; b++) {
       release(q->hdr[b]);
@@ -271,6 +306,16 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
             ensure(e->counts_dev, 16) == cudaSuccess && ensure(e->nmatched, 8) == cudaSuccess &&
             ensure(e->err, 4) == cudaSuccess && ensure(e->info, sizeof(SnapInfo)) == cudaSuccess;
   if (ok && semantics == MM_SEM_MPI) {
+    ok = cudaStreamCreateWithFlags(&e->cs, cudaStreamNonBlocking) == cudaSuccess &&
+         cudaStreamCreateWithFlags(&e->ds, cudaStreamNonBlocking) == cudaSuccess &&
+         cudaEventCreateWithFlags(&e->ev_st, cudaEventDisableTiming) == cudaSuccess &&
+         cudaMallocHost(&e->h_off, (size_t)(n_endpoints + 1) * 8) == cudaSuccess;
+    for (int k = 0; ok && k < kMaxChunks; k++)
+      ok = cudaEventCreateWithFlags(&e->ev_k[k], cudaEventDisableTiming) == cudaSuccess &&
+           cudaEventCreateWithFlags(&e->rq.ev[k], cudaEventDisableTiming) == cudaSuccess &&
+           cudaEventCreateWithFlags(&e->mq.ev[k], cudaEventDisableTiming) == cudaSuccess;
+  }
+  if (ok && semantics == MM_SEM_MPI) {
     e->msg_slots = (e->mcap + 63) / 64 * 64;
     e->warp_words = (e->msg_slots + e->msg_slots / 64 + 3) / 4 * 4;  // headers + availability bits, 32 B aligned
     e->fifo = fifo_layout(e->rcap, e->mcap);
@@ -316,8 +361,46 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
   return MM_OK;
 }
 
+// Submit the chunk copies of the deferred host inputs of queues qs[0..nq),
+// range by range (range k of every queue before range k + 1 of any).
+static int issue_chunks(mm_engine* e, Queue** qs, int nq) {
+  bool any = false;
+  for (int i = 0; i < nq; i++) any |= qs[i]->pend.active && qs[i]->pend.chunks > 0 && !qs[i]->pend.issued;
+  if (!any) return MM_OK;
+  CK(cudaEventRecord(e->ev_st, e->st));  // the staging buffers are free once earlier work on st is done
+  CK(cudaStreamWaitEvent(e->cs, e->ev_st, 0));
+  for (int k = 0; k < kMaxChunks; k++)
+    for (int i = 0; i < nq; i++) {
+      Pending& p = qs[i]->pend;
+      if (!p.active || p.chunks <= k || p.issued) continue;
+      const int64_t a = p.h_off[chunk_ep(e, k, p.chunks)], b = p.h_off[chunk_ep(e, k + 1, p.chunks)];
+      if (b > a) {
+        CK(cudaMemcpyAsync((uint64_t*)p.hdr + a, p.h_hdr + a, (size_t)(b - a) * 8, cudaMemcpyHostToDevice, e->cs));
+        if (p.h_cookie)
+          CK(cudaMemcpyAsync((int64_t*)p.cookie + a, p.h_cookie + a, (size_t)(b - a) * 8, cudaMemcpyHostToDevice,
+                             e->cs));
+      }
+      CK(cudaEventRecord(qs[i]->ev[k], e->cs));
+    }
+  for (int i = 0; i < nq; i++)
+    if (qs[i]->pend.active && qs[i]->pend.chunks > 0) qs[i]->pend.issued = true;
+  return MM_OK;
+}
+
+// Order the engine stream after every chunk copy of q's pending host input.
+static int join_pending(mm_engine* e, Queue& q) {
+  if (!q.pend.active || q.pend.chunks == 0) return MM_OK;
+  Queue* qs[1] = {&q};
+  int rc = issue_chunks(e, qs, 1);
+  if (rc != MM_OK) return rc;
+  CK(cudaStreamWaitEvent(e->st, q.ev[q.pend.chunks - 1], 0));
+  return MM_OK;
+}
+
 static int materialize(mm_engine* e, Queue& q, int64_t cap) {
   if (!q.pend.active) return MM_OK;
+  int jr = join_pending(e, q);
+  if (jr != MM_OK) return jr;
   Side s = make_side(e, q, cap);
   CK(launch_materialize(s, e->n_ep, (uint64_t*)q.hdr[q.cur].p, (int64_t*)q.cookie[q.cur].p, (int32_t*)q.len[q.cur].p,
                         (uint32_t*)e->err.p, e->st));
@@ -346,7 +429,23 @@ static int post(mm_engine* e, Queue& q, int64_t cap, const uint64_t* hdr, const 
   p.n = n;
   p.seq0 = q.seq;
   p.active = n > 0;
-  if (n > 0) {
+  const int C = pipeline_chunks(e);
+  if (n > 0 && C > 1 && off && !off_dev && !is_device_ptr(hdr) && (!cookie || !is_device_ptr(cookie))) {
+    // Host input of the MPI level: staged in endpoint ranges on the copy
+    // stream, submitted by mm_match_batch (issue_chunks) so that range k of
+    // both queues lands first and is matched while k + 1 is in flight.
+    CK(ensure(q.st_hdr, (size_t)n * 8));
+    if (cookie) CK(ensure(q.st_cookie, (size_t)n * 8));
+    CK(ensure(q.st_off, (size_t)(e->n_ep + 1) * 8));
+    CK(cudaMemcpyAsync(q.st_off.p, off, (size_t)(e->n_ep + 1) * 8, cudaMemcpyHostToDevice, e->st));
+    p.hdr = (const uint64_t*)q.st_hdr.p;
+    p.cookie = cookie ? (const int64_t*)q.st_cookie.p : nullptr;
+    p.off = (const int64_t*)q.st_off.p;
+    p.h_hdr = hdr;
+    p.h_cookie = cookie;
+    p.h_off = off;
+    p.chunks = C;
+  } else if (n > 0) {
     if (is_device_ptr(hdr)) {
       p.hdr = hdr;
     } else {
@@ -429,9 +528,31 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
     drc = (int64_t*)e->out_rc_stage.p;
     dmc = (int64_t*)e->out_mc_stage.p;
   }
+  // Host-buffer pipeline: endpoint range k runs once its H2D chunks landed,
+  // and its D2H starts as soon as it finished (H2D, kernels, D2H overlap).
+  const int C = pipeline_chunks(e);
+  const bool pipe = C > 1 && (host_out || e->rq.pend.chunks > 0 || e->mq.pend.chunks > 0);
+  Queue* qs[2] = {&e->rq, &e->mq};
+  if (pipe) {
+    Queue* pq[2];
+    int np = 0;
+    for (Queue* q : qs)
+      if (q->pend.chunks == C) pq[np++] = q;
+    int ir = issue_chunks(e, pq, np);
+    if (ir != MM_OK) return ir;
+  }
+  for (Queue* q : qs)
+    if (!pipe || q->pend.chunks != C) {
+      int jr = join_pending(e, *q);
+      if (jr != MM_OK) return jr;
+    }
   Side R = make_side(e, e->rq, e->rcap), M = make_side(e, e->mq, e->mcap);
   CK(cudaMemsetAsync(e->nmatched.p, 0, 8, e->st));
   CK(launch_out_offsets(R, e->n_ep, (int64_t*)e->out_off.p, out_cap, (uint32_t*)e->err.p, e->st));
+  if (host_out) {  // the output ranges are only known on the device: fetch them first
+    CK(cudaMemcpyAsync(e->h_off, e->out_off.p, (size_t)(e->n_ep + 1) * 8, cudaMemcpyDeviceToHost, e->st));
+    CK(cudaStreamSynchronize(e->st));
+  }
   MpiArgs a;
   a.R = R;
   a.M = M;
@@ -450,26 +571,42 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
   a.mres_w = (int32_t*)e->mq.len[0].p;
   a.n_matched = (unsigned long long*)e->nmatched.p;
   a.err = (uint32_t*)e->err.p;
+  const int nchunk = pipe ? C : 1;
   e->timer.begin(e->st);
-  if (e->mpi_kernel == MM_MPI_KERNEL_MATRIX)
-    CK(launch_mpi_matrix(a, e->st));
-  else
-    CK(launch_mpi_fifo(a, e->fifo, (uint8_t*)e->fifo_ws.p, e->st));
+  for (int k = 0; k < nchunk; k++) {
+    a.ep0 = (int)chunk_ep(e, k, nchunk);
+    a.n_ep = (int)chunk_ep(e, k + 1, nchunk);
+    if (pipe)
+      for (Queue* q : qs)
+        if (q->pend.active && q->pend.chunks == C) CK(cudaStreamWaitEvent(e->st, q->ev[k], 0));
+    if (e->mpi_kernel == MM_MPI_KERNEL_MATRIX)
+      CK(launch_mpi_matrix(a, e->st));
+    else
+      CK(launch_mpi_fifo(a, e->fifo, (uint8_t*)e->fifo_ws.p, e->st));
+    if (pipe && host_out) {
+      const int64_t o0 = e->h_off[a.ep0] < out_cap ? e->h_off[a.ep0] : out_cap;
+      const int64_t o1 = e->h_off[a.n_ep] < out_cap ? e->h_off[a.n_ep] : out_cap;
+      if (o1 > o0) {
+        CK(cudaEventRecord(e->ev_k[k], e->st));
+        CK(cudaStreamWaitEvent(e->ds, e->ev_k[k], 0));
+        CK(cudaMemcpyAsync(out_rc + o0, drc + o0, (size_t)(o1 - o0) * 8, cudaMemcpyDeviceToHost, e->ds));
+        CK(cudaMemcpyAsync(out_mc + o0, dmc + o0, (size_t)(o1 - o0) * 8, cudaMemcpyDeviceToHost, e->ds));
+      }
+    }
+  }
   e->timer.end(e->st);
   CK(launch_finalize((const int64_t*)e->out_off.p + e->n_ep, 0, (const unsigned long long*)e->nmatched.p,
                      (int64_t*)e->counts_dev.p, e->st));
   e->rq.pend = Pending();
   e->mq.pend = Pending();
   if (counts && !counts_host) CK(cudaMemcpyAsync(counts, e->counts_dev.p, 16, cudaMemcpyDeviceToDevice, e->st));
-  int64_t n_copy = 0;
-  if (host_out) {
-    // the snapshot size is only known on the device: fetch it first
-    int64_t tot = 0;
-    CK(cudaMemcpyAsync(&tot, (const int64_t*)e->out_off.p + e->n_ep, 8, cudaMemcpyDeviceToHost, e->st));
-    CK(cudaStreamSynchronize(e->st));
-    n_copy = tot < out_cap ? tot : out_cap;
+  if (pipe) CK(cudaStreamSynchronize(e->cs));  // the caller may reuse its host inputs once we return
+  if (pipe && host_out) {
+    CK(cudaStreamSynchronize(e->ds));
+    return deliver(e, out_rc, out_mc, false, 0, counts, counts_host);
   }
-  return deliver(e, out_rc, out_mc, host_out, n_copy, counts, counts_host);
+  const int64_t tot = e->h_off[e->n_ep];
+  return deliver(e, out_rc, out_mc, host_out, host_out ? (tot < out_cap ? tot : out_cap) : 0, counts, counts_host);
 }
 
 static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out_cap, int64_t* counts) {
@@ -609,6 +746,11 @@ int mm_set_option(mm_engine* e, int32_t option, int64_t value) {
   if (option == MM_OPT_FLAT_KERNEL) {
     if (value != MM_FLAT_KERNEL_BUCKETED && value != MM_FLAT_KERNEL_GLOBAL) return MM_ERR_ARG;
     e->flat_kernel = (int)value;
+    return MM_OK;
+  }
+  if (option == MM_OPT_PIPELINE_CHUNKS) {
+    if (value < 0 || value > kMaxChunks) return MM_ERR_ARG;
+    e->pipeline = (int)value;
     return MM_OK;
   }
   if (option == MM_OPT_MPI_KERNEL) {

@@ -7,7 +7,8 @@ namespace mm {
 
 struct MpiArgs {
   Side R, M;
-  int n_ep;
+  int n_ep;      // endpoints [ep0, n_ep) are matched by this launch
+  int ep0 = 0;
   int64_t msg_slots;        // shared-memory message slots per warp (>= msg cap, multiple of 64)
   int64_t warp_smem_words;  // 8-byte words of shared memory per warp
   int64_t* out_rc;

@@ -17,27 +17,36 @@ def to_dev(a):
     return torch.from_numpy(a.copy()).cuda()
 
 
-def gpu_batches(sem, n_ep, rcap, mcap, batches, host=False, out_cap=None, mpi_kernel=None, flat_kernel=None):
+def gpu_batches(sem, n_ep, rcap, mcap, batches, host=False, out_cap=None, mpi_kernel=None, flat_kernel=None,
+                pipeline=None):
     """batches: list of (recv_hdr, recv_cookie, recv_off, msg_hdr, msg_cookie, msg_off).
+    host: False (device buffers), True (host inputs and outputs), "in" (host
+    inputs, device outputs) or "out" (device inputs, host outputs).
+    pipeline: MM_OPT_PIPELINE_CHUNKS value (None = engine default).
     Returns a list of (out_rc, out_mc) numpy arrays, one per batch."""
     import torch
     from paper_conf_ipps_klenkfed17_b200 import Engine
+    from paper_conf_ipps_klenkfed17_b200._lib import MM_OPT_PIPELINE_CHUNKS
     eng = Engine(sem, n_ep, rcap, mcap, mpi_kernel=mpi_kernel, flat_kernel=flat_kernel)
+    if pipeline is not None:
+        eng.set_option(MM_OPT_PIPELINE_CHUNKS, pipeline)
+    host_in = host is True or host == "in"
+    host_out = host is True or host == "out"
     res = []
     for (rh, rc, ro, mh, mc, mo) in batches:
-        if host:
+        if host_in:
             eng.post_recvs(np.ascontiguousarray(rh, np.uint64), rc, ro)
             eng.push_msgs(np.ascontiguousarray(mh, np.uint64), mc, mo)
         else:
             eng.post_recvs(to_dev(rh), to_dev(rc), to_dev(ro))
             eng.push_msgs(to_dev(mh), to_dev(mc), to_dev(mo))
         cap = out_cap if out_cap is not None else n_ep * rcap
-        if host:
+        if host_out:
             orc = np.full(cap, -7, np.int64)
             omc = np.full(cap, -7, np.int64)
             cnt = np.zeros(2, np.int64)
             eng.match_batch(orc, omc, cnt)
-            n = int(cnt[0])
+            n = min(int(cnt[0]), cap)
             res.append((orc[:n].copy(), omc[:n].copy(), cnt.copy()))
         else:
             orc = torch.full((cap,), -7, dtype=torch.int64, device="cuda")
@@ -46,7 +55,7 @@ def gpu_batches(sem, n_ep, rcap, mcap, batches, host=False, out_cap=None, mpi_ke
             eng.match_batch(orc, omc, cnt)
             torch.cuda.synchronize()
             c = cnt.cpu().numpy()
-            n = int(c[0])
+            n = min(int(c[0]), cap)
             res.append((orc[:n].cpu().numpy(), omc[:n].cpu().numpy(), c))
     q = eng.query(raise_on_error=False)
     eng.close()

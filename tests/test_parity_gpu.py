@@ -92,6 +92,40 @@ def test_mpi_host_buffers_equal_device(kern):
     assert_exact(gh, o)
 
 
+@pytest.mark.parametrize("chunks", [0, 1, 2, 3, 7, 32])
+@pytest.mark.parametrize("host", [True, "in", "out"], ids=["host-io", "host-in", "host-out"])
+@KERNELS
+def test_mpi_host_pipeline(chunks, host, kern):
+    """Host-buffer pipeline (MM_OPT_PIPELINE_CHUNKS): endpoint ranges copied in,
+    matched and copied out on three streams; 3 batches with residuals, user
+    cookies, ragged and empty endpoints -- identical to the oracle for every
+    range count."""
+    rng = np.random.default_rng(chunks)
+    q = synth.mpi_endpoints(40 + chunks, n_ep=301, depth_r=96, n_src=6, n_tag=4, p_any_src=0.2, p_any_tag=0.1,
+                            ragged=True, p_unmatched=0.25)
+    batches = split_batches(q, 3, rng)  # carries user cookies (global element ids)
+    g, qs = gpu_batches(MPI, q.n_endpoints, 300, 300, batches, host=host, mpi_kernel=kern, pipeline=chunks)
+    o, oe = oracle_batches(MPI, q.n_endpoints, batches)
+    assert_exact(g, o)
+    rr, rm = oe.residual_depths()
+    assert qs["error"] == 0 and qs["resid_recv"] == sum(rr) and qs["resid_msg"] == sum(rm)
+
+
+def test_mpi_host_pipeline_truncated_output():
+    """A host output too small for the snapshot: the capacity flag is raised
+    and the copied prefix is still the oracle's."""
+    q = synth.mpi_endpoints(77, n_ep=260, depth_r=64, ragged=True, p_unmatched=0.1)
+    o, _ = oracle_batches(MPI, q.n_endpoints, single_batch(q))
+    cap = len(o[0][0]) // 2
+    g, qs = gpu_batches(MPI, q.n_endpoints, 64, 64, single_batch(q), host=True, out_cap=cap, pipeline=4)
+    assert qs["error"] != 0
+    # endpoints whose output range fits are reported exactly; the rest is
+    # flagged and its output positions are unspecified
+    fit = int(q.recv_off[np.searchsorted(q.recv_off, cap, side="right") - 1])
+    assert fit > 0
+    assert np.array_equal(g[0][0][:fit], o[0][0][:fit]) and np.array_equal(g[0][1][:fit], o[0][1][:fit])
+
+
 @KERNELS
 def test_mpi_user_cookies_and_two_posts(kern):
     """Cookies are carried through; a second post before a match is queued."""

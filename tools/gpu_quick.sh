@@ -9,5 +9,5 @@ else timeout 900 python -m pytest tests -m gpu -q -x -p no:cacheprovider > gpuru
 tail -3 gpurun_out/pytest_$TAG.log; grep -m5 -B5 "Error\|assert" gpurun_out/pytest_$TAG.log | head -60
 timeout 600 python bench.py --levels $LV --no-cpu-baseline > gpurun_out/bench_$TAG.log 2>&1; tail -1 gpurun_out/bench_$TAG.log | python -c "
 import json,sys; d=json.loads(sys.stdin.read())
-for k,v in d['levels'].items(): print(k, round(v['value']/1e9,3), 'Gm/s', round(v['ms_per_step'],3), 'ms kernel', round(v['roofline']['kernel_ms'],3), 'frac', round(v['roofline']['frac'],4))" || tail -5 gpurun_out/bench_$TAG.log
+for k,v in d['levels'].items(): print(k, round(v['value']/1e9,3), 'Gm/s', round(v['ms_per_step'],3), 'ms kernel', round(v['roofline']['kernel_ms'],3), 'frac', round(v['roofline']['frac'],4), 'e2e', round(v['e2e']['value']/1e9,3) if 'e2e' in v else '', v.get('e2e',{}).get('ms_per_step',''))" || tail -5 gpurun_out/bench_$TAG.log
 if [ -n "$PHASE" ]; then python -c "from paper_conf_ipps_klenkfed17_b200 import _build; _build.build_library(variant='timing')" && python tools/phase_timing.py 2>&1 | tail -16; fi
