@@ -82,7 +82,9 @@ enum {
                             (NOWILD_ORDERED), the hash kernels (NOWILD_UNORDERED) */
     MM_Q_KERNEL_RUNS = 6,/* number of timed regions behind MM_Q_KERNEL_NS */
     MM_Q_LAUNCHES = 7,   /* cumulative count of this library's kernel launches */
-    MM_Q_COUNT = 8
+    MM_Q_FALLBACKS = 8,  /* no-wildcard batches that overflowed a bucket and ran the
+                            global kernels instead */
+    MM_Q_COUNT = 9
 };
 
 typedef struct mm_engine mm_engine; /* opaque, owned by the library */

@@ -34,7 +34,7 @@ MM_ANY_TAG = 0xFFFF
 MM_MPI_MAX_MSGS = 24576
 
 (MM_Q_N_OUT, MM_Q_N_MATCHED, MM_Q_RESID_RECV, MM_Q_RESID_MSG, MM_Q_ERROR, MM_Q_KERNEL_NS, MM_Q_KERNEL_RUNS,
- MM_Q_LAUNCHES, MM_Q_COUNT) = range(9)
+ MM_Q_LAUNCHES, MM_Q_FALLBACKS, MM_Q_COUNT) = range(10)
 
 # name -> (restype, argtypes); must list every function include/mm.h declares
 _P = ctypes.c_void_p

@@ -9,15 +9,16 @@
 //     bits, 8 bits per pass) -- stability keeps posting / arrival order inside
 //     every bucket;
 //  2. match every bucket in one CTA, entirely in shared memory: message tuples
-//     go into a lock-free open-addressing hash table (16-bit CAS), receives
-//     look their tuple up, and each element gets its rank among the equal
-//     tuples of its side:
-//       - NOWILD_ORDERED: ranks in posting / arrival order (warp-ordered
-//         placement, quarters in parallel) -- the n-th receive of a tuple takes
-//         the n-th message of it, the MPI result without wildcards;
-//       - NOWILD_UNORDERED: ranks from shared-memory atomics, any order -- a
-//         maximal pairing of equal tuples, what the relaxation allows;
-//     the receive of rank r pairs with the message of rank r;
+//     get dense ids from a lock-free open-addressing table (32-bit CAS),
+//     receives look their tuple up, and
+//       - NOWILD_ORDERED (k_bucket_pair, persistent CTAs): every element gets
+//         its rank among the equal tuples of its side in posting / arrival
+//         order (quarters walked by one warp each with match.any peers) --
+//         the receive of rank r takes the message of rank r, the MPI result
+//         without wildcards;
+//       - NOWILD_UNORDERED (k_bucket_pop): messages are pushed onto per-tuple
+//         lists and receives pop from them -- a maximal pairing of equal
+//         tuples, what the relaxation allows;
 //  3. write results at the elements' snapshot positions and matched flags for
 //     the queue compaction.
 // A bucket larger than the on-chip capacity raises a flag; the host then runs
@@ -170,7 +171,7 @@ static cudaError_t partition_side(const SnapRead& snap, int64_t n, int nb, uint6
 constexpr int kBucketCap = 1024;   // elements (receives + messages) per bucket on chip
 constexpr int kBucketThreads = 256;
 constexpr uint32_t kBucketH = 2048;  // hash slots (>= 2 * kBucketCap)
-constexpr uint32_t kMaxRun = 64;     // ordered: longest run of one tuple walked on chip
+constexpr int kQ = 4;                // ordered: quarters per side, ranked by one warp each
 
 struct BucketArgs {
   FlatArgs a;
@@ -185,26 +186,256 @@ struct BucketArgs {
 
 // Elements of a bucket are kept in snapshot order (the partition is stable),
 // so an element's bucket position orders it among the equal tuples of its
-// side.  Tuples are found through an open-addressing table of 32-bit entries
-// (16-bit fingerprint | representative element); the elements of a tuple form
-// singly linked lists per side, pushed with one atomic exchange each.
-template <bool ORDERED>
+// side.  Message tuples get dense ids through an open-addressing table of
+// 32-bit entries (16-bit fingerprint | representative element; the CAS winner
+// draws the id).  Every element then gets its rank among the equal tuples of
+// its side in bucket order: each side is cut in kQ quarters, one warp per
+// quarter walks it 32 elements at a time (match.any peers, per-tuple running
+// counts), then per-tuple prefixes over the quarters complete the ranks.
+// Messages are placed by (tuple, rank) after a scan of the per-tuple message
+// counts, and the receive of rank r takes the message of rank r of its tuple.
+// O(1) work per element (no list walks, no run-length limit), 7 barriers.
 struct BucketSmem {
+  uint64_t hdr[kBucketCap];  // receives [0, nr), then messages [nr, nr + nm)
+  uint32_t idx[kBucketCap];  // snapshot index
+  uint32_t table[kBucketH];  // tuple table
+  uint16_t sid[kBucketH];    // slot -> dense tuple id (valid where table[slot] is set)
+  uint16_t tup[kBucketCap];  // element -> slot (messages, phase B), then tuple id | kNone
+  uint16_t rnk[kBucketCap];  // element -> rank among its side's equal tuples
+  // qcnt[side][quarter][tuple]: running counts, then exclusive prefixes over
+  // the quarters
+  uint16_t qcnt[2 * kQ * kBucketCap];
+  uint16_t mstart[kBucketCap];  // tuple -> first position in msg_at
+  uint16_t mtot[kBucketCap];    // tuple -> number of messages
+  uint16_t msg_at[kBucketCap];  // messages grouped by tuple, in rank order
+  uint32_t matched[kBucketCap / 32];
+  uint32_t scan_sm[kBucketThreads / 32 + 1];
+  uint32_t ntup;
+};
+
+// quarter of position x in a side of length L (boundaries q * L / kQ)
+__device__ __forceinline__ uint32_t quarter_of(uint32_t x, uint32_t L) {
+  return (uint32_t)(x >= L / 4) + (uint32_t)(x >= L / 2) + (uint32_t)(x >= (3 * L) / 4);
+}
+
+__global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba, uint32_t nbk) {
+  extern __shared__ __align__(16) uint8_t smem_raw[];
+  BucketSmem& sm = *reinterpret_cast<BucketSmem*>(smem_raw);
+  constexpr int NT = kBucketThreads;
+  constexpr int PER = kBucketCap / NT;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const FlatArgs& a = ba.a;
+  const int64_t rres = a.R.q_len[0], rpb = a.R.pend_begin(0);
+  const int64_t mres = a.M.q_len[0], mpb = a.M.pend_begin(0);
+  constexpr uint32_t hmask = kBucketH - 1;
+  // Persistent: buckets blockIdx.x, + gridDim.x, ...; the next bucket's
+  // elements are loaded into registers while the current one is matched.
+  uint64_t hv[PER];
+  uint32_t iv[PER];
+  auto fetch = [&](uint32_t bb, uint32_t& fr0, uint32_t& fnr, uint32_t& fm0, uint32_t& fnm) {
+    fr0 = fnr = fm0 = fnm = 0;
+    if (bb < nbk) {
+      fr0 = ba.roff[bb];
+      fnr = ba.roff[bb + 1] - fr0;
+      fm0 = ba.moff[bb];
+      fnm = ba.moff[bb + 1] - fm0;
+    }
+    const bool fits = fnr + fnm <= (uint32_t)kBucketCap;
+#pragma unroll
+    for (int u = 0; u < PER; u++) {
+      const uint32_t e = tid + u * NT;
+      hv[u] = 0;
+      iv[u] = 0;
+      if (fits && e < fnr) {
+        hv[u] = ba.rh[fr0 + e];
+        iv[u] = (uint32_t)ba.ri[fr0 + e];
+      } else if (fits && e < fnr + fnm) {
+        hv[u] = ba.mh[fm0 + e - fnr];
+        iv[u] = (uint32_t)ba.mi[fm0 + e - fnr];
+      }
+    }
+  };
+  uint32_t xr0, xnr, xm0, xnm;  // bounds of the bucket held in hv / iv
+  fetch(blockIdx.x, xr0, xnr, xm0, xnm);
+  for (uint32_t b = blockIdx.x; b < nbk; b += gridDim.x) {
+    __syncthreads();  // the previous bucket is done with shared memory
+    const uint32_t r0 = xr0, nr = xnr, m0 = xm0, nm = xnm;
+    const uint32_t n = nr + nm;
+    if (n == 0 || n > (uint32_t)kBucketCap) {  // uniform across the CTA
+      if (n > (uint32_t)kBucketCap && tid == 0) atomicOr(ba.overflow, 1u);
+      fetch(b + gridDim.x, xr0, xnr, xm0, xnm);
+      continue;
+    }
+    // A: registers to shared memory, clear the tables, prefetch the next bucket
+#pragma unroll
+    for (int u = 0; u < PER; u++) {
+      const uint32_t e = tid + u * NT;
+      if (e < n) {
+        sm.hdr[e] = hv[u];
+        sm.idx[e] = iv[u];
+      }
+    }
+    for (uint32_t s = tid; s < kBucketH / 4; s += NT) reinterpret_cast<uint4*>(sm.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
+    if (tid < kBucketCap / 32) sm.matched[tid] = 0u;
+    if (tid == 0) sm.ntup = 0;
+    fetch(b + gridDim.x, xr0, xnr, xm0, xnm);
+  __syncthreads();
+  // B: message tuples into the table; the CAS winner draws the dense id
+  for (uint32_t e = nr + tid; e < n; e += NT) {
+    const uint64_t h = sm.hdr[e];
+    const uint64_t p = h * 0xD6E8FEB86659FD93ull;
+    uint32_t s = (uint32_t)(p >> 40) & hmask;
+    const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
+    while (true) {
+      uint32_t o = sm.table[s];
+      if (o == 0xFFFFFFFFu) {
+        o = atomicCAS(&sm.table[s], 0xFFFFFFFFu, (fp << 16) | e);  // representative's header is in smem already
+        if (o == 0xFFFFFFFFu) {
+          sm.sid[s] = (uint16_t)atomicAdd(&sm.ntup, 1u);
+          break;
+        }
+      }
+      if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) break;
+      s = (s + 1) & hmask;
+    }
+    sm.tup[e] = (uint16_t)s;
+  }
+  __syncthreads();
+  const uint32_t T = sm.ntup;
+  // C: tuple ids (receives look theirs up) and ranks within the side
+  {
+    const uint32_t side = warp < kQ ? 1u : 0u, q = warp & (kQ - 1);
+    uint16_t* run = &sm.qcnt[(side * kQ + q) * kBucketCap];
+    for (uint32_t t = lane; t < T; t += 32) run[t] = 0;
+    __syncwarp();
+    const uint32_t L = side ? nm : nr, base = side ? nr : 0u;
+    const uint32_t lo = base + (q * L) / kQ, hi = base + ((q + 1) * L) / kQ;
+    const uint32_t lt = lanemask_lt();
+    for (uint32_t c = lo; c < hi; c += 32) {
+      const uint32_t e = c + lane;
+      uint32_t id = kNone;
+      if (e < hi) {
+        if (side) {
+          id = sm.sid[sm.tup[e]];
+        } else {
+          const uint64_t h = sm.hdr[e];
+          const uint64_t p = h * 0xD6E8FEB86659FD93ull;
+          uint32_t s = (uint32_t)(p >> 40) & hmask;
+          const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
+          while (true) {
+            const uint32_t o = sm.table[s];
+            if (o == 0xFFFFFFFFu) break;
+            if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) {
+              id = sm.sid[s];
+              break;
+            }
+            s = (s + 1) & hmask;
+          }
+        }
+      }
+      const bool has = id != kNone;
+      const uint32_t peers = __match_any_sync(kFull, has ? id : 0x10000u + lane);
+      const uint32_t before = has ? run[id] : 0u;
+      __syncwarp();
+      if (has && (peers >> lane) == 1u) run[id] = (uint16_t)(before + __popc(peers));  // highest peer publishes
+      if (e < hi) {
+        sm.tup[e] = (uint16_t)id;
+        sm.rnk[e] = (uint16_t)(before + __popc(peers & lt));
+      }
+      __syncwarp();
+    }
+  }
+  __syncthreads();
+  // D: per tuple -- prefixes over the quarters, message totals, and their
+  // scan (tuples 4 * tid .. 4 * tid + 3)
+  {
+    uint32_t tot[4], sum = 0;
+#pragma unroll
+    for (int j = 0; j < 4; j++) {
+      const uint32_t t = 4 * tid + j;
+      tot[j] = 0;
+      if (t < T) {
+#pragma unroll
+        for (int side = 0; side < 2; side++) {
+          uint32_t acc = 0;
+#pragma unroll
+          for (int q = 0; q < kQ; q++) {
+            uint16_t* c = &sm.qcnt[(side * kQ + q) * kBucketCap + t];
+            const uint32_t v = *c;
+            *c = (uint16_t)acc;
+            acc += v;
+          }
+          if (side) tot[j] = acc;
+        }
+      }
+      sum += tot[j];
+    }
+    uint32_t all;
+    uint32_t ex = block_excl_scan<uint32_t>(sum, sm.scan_sm, &all);
+#pragma unroll
+    for (int j = 0; j < 4; j++) {
+      const uint32_t t = 4 * tid + j;
+      if (t < T) {
+        sm.mstart[t] = (uint16_t)ex;
+        sm.mtot[t] = (uint16_t)tot[j];
+      }
+      ex += tot[j];
+    }
+  }
+  __syncthreads();
+  // E: full ranks; messages placed by (tuple, rank)
+  for (uint32_t e = tid; e < n; e += NT) {
+    const uint32_t id = sm.tup[e];
+    if (id == kNone) continue;
+    const uint32_t side = e >= nr ? 1u : 0u;
+    const uint32_t q = side ? quarter_of(e - nr, nm) : quarter_of(e, nr);
+    const uint32_t r = sm.rnk[e] + sm.qcnt[(side * kQ + q) * kBucketCap + id];
+    if (!side) sm.rnk[e] = (uint16_t)r;
+    if (e >= nr) sm.msg_at[sm.mstart[id] + r] = (uint16_t)e;
+  }
+  __syncthreads();
+  // F: receives take the message of equal rank
+  uint32_t nmatch = 0;
+  for (uint32_t e = tid; e < nr; e += NT) {
+    const uint32_t id = sm.tup[e];
+    uint32_t j = kNone;
+    if (id != kNone) {
+      const uint32_t r = sm.rnk[e];
+      if (r < sm.mtot[id]) j = sm.msg_at[sm.mstart[id] + r];
+    }
+    int64_t mc = MM_NO_MATCH;
+    if (j != kNone) {
+      atomicOr(&sm.matched[(j - nr) >> 5], 1u << ((j - nr) & 31));
+      mc = a.M.cookie(0, sm.idx[j], mres, mpb);
+      nmatch++;
+    }
+    a.out_rc[r0 + e] = a.R.cookie(0, sm.idx[e], rres, rpb);
+    a.out_mc[r0 + e] = mc;
+    a.rflag[r0 + e] = j != kNone ? 1 : 0;
+  }
+  for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
+  if (lane == 0 && nmatch) atomicAdd(a.n_matched, (unsigned long long)nmatch);
+  __syncthreads();
+  for (uint32_t x = tid; x < nm; x += NT) a.mflag[m0 + x] = (sm.matched[x >> 5] >> (x & 31)) & 1u;
+  }
+}
+
+// NOWILD_UNORDERED: messages pushed onto per-tuple lists, receives pop from
+// them (lock-free, pops only in that phase: no ABA) -- any maximal pairing of
+// equal tuples; 3 barriers.
+struct PopSmem {
   uint64_t hdr[kBucketCap];               // receives [0, nr), then messages [nr, nr + nm)
   uint32_t idx[kBucketCap];               // snapshot index
   uint32_t table[kBucketH];               // tuple table
   uint16_t mhead[kBucketH];               // per slot: message list
-  uint16_t rhead[ORDERED ? kBucketH : 2];  // per slot: receive list (ordered)
   uint16_t next[kBucketCap];              // list links
   uint16_t slot[kBucketCap];              // receive -> slot | kNone
-  uint16_t rank[ORDERED ? kBucketCap : 2];  // message rank among its tuple's messages
   uint32_t matched[kBucketCap / 32];      // message matched bits (by message offset)
 };
 
-template <bool ORDERED>
-__global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
+__global__ void __launch_bounds__(kBucketThreads) k_bucket_pop(BucketArgs ba) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
-  BucketSmem<ORDERED>& sm = *reinterpret_cast<BucketSmem<ORDERED>*>(smem_raw);
+  PopSmem& sm = *reinterpret_cast<PopSmem*>(smem_raw);
   constexpr int NT = kBucketThreads;
   const int tid = threadIdx.x, lane = tid & 31;
   const FlatArgs& a = ba.a;
@@ -239,8 +470,6 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
     }
     for (uint32_t s = tid; s < kBucketH / 4; s += NT) reinterpret_cast<uint4*>(sm.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
     for (uint32_t s = tid; s < kBucketH / 8; s += NT) reinterpret_cast<uint4*>(sm.mhead)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
-    if (ORDERED)
-      for (uint32_t s = tid; s < kBucketH / 8; s += NT) reinterpret_cast<uint4*>(sm.rhead)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
     for (uint32_t s = tid; s < kBucketCap / 32; s += NT) sm.matched[s] = 0u;
 #pragma unroll
     for (int u = 0; u < PER; u++) {
@@ -270,7 +499,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
     sm.next[e] = exch16(&sm.mhead[s], (uint16_t)e);
   }
   __syncthreads();
-  // receives: look the tuple up (ordered: push onto its receive list)
+  // receives: look the tuple up
   for (uint32_t e = tid; e < nr; e += NT) {
     const uint64_t h = sm.hdr[e];
     const uint64_t p = h * 0xD6E8FEB86659FD93ull;
@@ -287,53 +516,22 @@ __global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba) {
       s = (s + 1) & hmask;
     }
     sm.slot[e] = (uint16_t)found;
-    if (ORDERED && found != kNone) sm.next[e] = exch16(&sm.rhead[found], (uint16_t)e);
-  }
-  if (ORDERED) {
-    // message ranks: earlier messages of the same tuple have smaller positions
-    for (uint32_t e = nr + tid; e < n; e += NT) {
-      const uint64_t h = sm.hdr[e];
-      const uint64_t p = h * 0xD6E8FEB86659FD93ull;
-      uint32_t s = (uint32_t)(p >> 40) & hmask;
-      const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
-      while (true) {
-        const uint32_t o = sm.table[s];
-        if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) break;
-        s = (s + 1) & hmask;
-      }
-      uint32_t r = 0, len = 0;
-      for (uint32_t x = sm.mhead[s]; x != kNone && len <= kMaxRun; x = sm.next[x], len++) r += x < e;
-      if (len > kMaxRun) atomicOr(ba.overflow, 1u);  // a tuple too long to rank by walking
-      sm.rank[e] = (uint16_t)r;
-    }
   }
   __syncthreads();
-  // receives take their message: ordered -- the message of equal rank;
-  // unordered -- any message of the tuple (pop from the list)
+  // receives take any message of their tuple (pop from the list)
   uint32_t nmatch = 0;
   for (uint32_t e = tid; e < nr; e += NT) {
     const uint32_t s = sm.slot[e];
     uint32_t j = kNone;
     if (s != kNone) {
-      if (ORDERED) {
-        uint32_t r = 0, len = 0;
-        for (uint32_t x = sm.rhead[s]; x != kNone && len <= kMaxRun; x = sm.next[x], len++) r += x < e;
-        if (len > kMaxRun) atomicOr(ba.overflow, 1u);
-        for (uint32_t x = sm.mhead[s]; x != kNone; x = sm.next[x])
-          if (sm.rank[x] == r) {
-            j = x;
-            break;
-          }
-      } else {
-        uint32_t hd = sm.mhead[s];
-        while (hd != kNone) {  // pops only in this phase: no ABA
-          const uint32_t got = cas16(&sm.mhead[s], (uint16_t)hd, sm.next[hd]);
-          if (got == hd) {
-            j = hd;
-            break;
-          }
-          hd = got;
+      uint32_t hd = sm.mhead[s];
+      while (hd != kNone) {  // pops only in this phase: no ABA
+        const uint32_t got = cas16(&sm.mhead[s], (uint16_t)hd, sm.next[hd]);
+        if (got == hd) {
+          j = hd;
+          break;
         }
+        hd = got;
       }
     }
     int64_t mc = MM_NO_MATCH;
@@ -360,6 +558,20 @@ int64_t bucket_bits_for(int64_t n) {
   return nb;
 }
 
+// persistent grid: every resident CTA slot of the chip, at most one per bucket
+template <class K>
+static uint32_t bucket_grid(K kernel, size_t smem, uint32_t B) {
+  int dev = 0, sms = 148, occ = 1;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess ||
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, kBucketThreads, smem) != cudaSuccess) {
+    cudaGetLastError();
+    sms = 148;
+    occ = 1;
+  }
+  const uint32_t g = (uint32_t)(sms * (occ < 1 ? 1 : occ));
+  return g < B ? g : B;
+}
+
 cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cudaStream_t st) {
   const int nb = (int)bucket_bits_for(a.nr + a.nm);
   const uint32_t B = 1u << nb;
@@ -378,17 +590,17 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cuda
   s.mi_sorted = mi;
   BucketArgs ba{a, rh, ri, s.roff, mh, mi, s.moff, s.overflow};
   if (ordered) {
-    const size_t smem = sizeof(BucketSmem<true>);
-    err = cudaFuncSetAttribute(k_bucket_pair<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const size_t smem = sizeof(BucketSmem);
+    err = cudaFuncSetAttribute(k_bucket_pair, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (err != cudaSuccess) return err;
     count_launch();
-    k_bucket_pair<true><<<B, kBucketThreads, smem, st>>>(ba);
+    k_bucket_pair<<<bucket_grid(k_bucket_pair, smem, B), kBucketThreads, smem, st>>>(ba, B);
   } else {
-    const size_t smem = sizeof(BucketSmem<false>);
-    err = cudaFuncSetAttribute(k_bucket_pair<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const size_t smem = sizeof(PopSmem);
+    err = cudaFuncSetAttribute(k_bucket_pop, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (err != cudaSuccess) return err;
     count_launch();
-    k_bucket_pair<false><<<B, kBucketThreads, smem, st>>>(ba);
+    k_bucket_pop<<<B, kBucketThreads, smem, st>>>(ba);
   }
   return cudaGetLastError();
 }

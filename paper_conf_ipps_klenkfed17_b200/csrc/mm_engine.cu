@@ -786,6 +786,7 @@ int mm_query(mm_engine* e, int64_t* vals) {
   vals[MM_Q_KERNEL_NS] = e->timer.ns;
   vals[MM_Q_KERNEL_RUNS] = e->timer.runs;
   vals[MM_Q_LAUNCHES] = e->launches;
+  vals[MM_Q_FALLBACKS] = e->bucket_fallbacks;
   if (e->sem != MM_SEM_MPI) {
     e->rq.resid_host = rsum;
     e->mq.resid_host = msum;

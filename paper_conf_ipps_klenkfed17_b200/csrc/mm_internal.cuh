@@ -227,7 +227,7 @@ inline int64_t scan_scratch_elems(int64_t n) { return (n + kScanTile - 1) / kSca
 // stable without CTA-wide barriers inside the tile.
 constexpr int kPartWarps = 8;
 constexpr int kPartThreads = kPartWarps * 32;
-constexpr int kPartItems = 8;                           // per lane
+constexpr int kPartItems = 6;                           // per lane
 constexpr int kPartMaxBuckets = 512;
 constexpr int kPartWarpChunk = 32 * kPartItems;         // 256 elements per warp
 constexpr int kPartTile = kPartWarps * kPartWarpChunk;  // 2048 elements per tile

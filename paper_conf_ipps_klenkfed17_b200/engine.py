@@ -129,7 +129,7 @@ class Engine:
             check(rc, "mm_query")
         return {"n_out": int(vals[0]), "n_matched": int(vals[1]), "resid_recv": int(vals[2]),
                 "resid_msg": int(vals[3]), "error": int(vals[4]), "kernel_ns": int(vals[5]),
-                "kernel_runs": int(vals[6]), "launches": int(vals[7]), "rc": rc}
+                "kernel_runs": int(vals[6]), "launches": int(vals[7]), "fallbacks": int(vals[8]), "rc": rc}
 
     def close(self):
         if getattr(self, "_h", None) is not None and self._h.value:

@@ -267,6 +267,25 @@ def test_ordered_all_same_key(flat):
     assert_same_pairs(g, o)
 
 
+def test_ordered_long_runs_stay_on_chip():
+    """Tuples repeated hundreds of times inside one bucket are ranked on chip
+    (O(1) per element, no run-length limit): bit-exact, no global fallback."""
+    rng = np.random.default_rng(11)
+    n = 8000
+    src = rng.integers(0, 1 << 20, n)
+    tag = rng.integers(0, 64, n)
+    src[rng.choice(n, 200, replace=False)] = 7  # one hot tuple (7, 3), 200 deep on each side
+    hot = src == 7
+    tag[hot] = 3
+    rh = synth.pack(src, tag)
+    mh = rh[rng.permutation(n)]
+    b = [(rh, None, np.array([0, n]), mh, None, np.array([0, n]))]
+    g, qs = gpu_batches(ORD, 1, n, n, b, flat_kernel=0)
+    o, _ = oracle_batches(ORD, 1, b)
+    assert_same_pairs(g, o)
+    assert qs["fallbacks"] == 0
+
+
 @pytest.mark.slow
 @FLAT
 def test_ordered_config2_full(flat):
