@@ -198,27 +198,34 @@ struct BucketArgs {
 struct BucketSmem {
   uint64_t hdr[kBucketCap];  // receives [0, nr), then messages [nr, nr + nm)
   uint32_t idx[kBucketCap];  // snapshot index
-  uint32_t table[kBucketH];  // tuple table
-  uint16_t sid[kBucketH];    // slot -> dense tuple id (valid where table[slot] is set)
+  union {
+    struct {                     // phases A..C
+      uint32_t table[kBucketH];  // tuple table
+      uint16_t sid[kBucketH];    // slot -> dense tuple id (valid where table[slot] is set)
+    };
+    struct {                        // phases D..F
+      uint16_t mstart[kBucketCap];  // tuple -> first position in msg_at
+      uint16_t mtot[kBucketCap];    // tuple -> number of messages
+      uint16_t msg_at[kBucketCap];  // messages grouped by tuple, in rank order
+    };
+  };
   uint16_t tup[kBucketCap];  // element -> slot (messages, phase B), then tuple id | kNone
   uint16_t rnk[kBucketCap];  // element -> rank among its side's equal tuples
   // qcnt[side][quarter][tuple]: running counts, then exclusive prefixes over
   // the quarters
   uint16_t qcnt[2 * kQ * kBucketCap];
-  uint16_t mstart[kBucketCap];  // tuple -> first position in msg_at
-  uint16_t mtot[kBucketCap];    // tuple -> number of messages
-  uint16_t msg_at[kBucketCap];  // messages grouped by tuple, in rank order
   uint32_t matched[kBucketCap / 32];
   uint32_t scan_sm[kBucketThreads / 32 + 1];
   uint32_t ntup;
 };
+static_assert(sizeof(BucketSmem) <= 44 * 1024 + 512, "five CTAs per SM");
 
 // quarter of position x in a side of length L (boundaries q * L / kQ)
 __device__ __forceinline__ uint32_t quarter_of(uint32_t x, uint32_t L) {
   return (uint32_t)(x >= L / 4) + (uint32_t)(x >= L / 2) + (uint32_t)(x >= (3 * L) / 4);
 }
 
-__global__ void __launch_bounds__(kBucketThreads) k_bucket_pair(BucketArgs ba, uint32_t nbk) {
+__global__ void __launch_bounds__(kBucketThreads, 5) k_bucket_pair(BucketArgs ba, uint32_t nbk) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   BucketSmem& sm = *reinterpret_cast<BucketSmem*>(smem_raw);
   constexpr int NT = kBucketThreads;

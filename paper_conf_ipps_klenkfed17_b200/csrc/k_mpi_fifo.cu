@@ -259,19 +259,22 @@ __device__ __forceinline__ void stream_chain(const FifoWs& ws, uint32_t* kmask, 
   if (own) ws.key_c[lane] = (uint16_t)c;
 }
 
-// The wildcard chain in its leanest form (about twenty instructions a step).
-// Lane l owns tuple k (own) and keeps, in registers, its next exact receive's
-// posting position (npos) and a window h0/h1 = list_k[cur + c], list_k[cur +
-// c + 1] of its message list: an exact receive of k posted before the
-// wildcard (cur++) and a win (c++) both shift the window by one.  Wildcards
-// are served in posting order from wl[x_begin..W) -- those with in(y) --, 32
-// positions at a time held in registers; `left` of them in all.  A step is a
-// shuffle, the cursor compare, one redux.sync.min and, for the winner, a
-// store and the window shift.  ADMIT: wildcards may differ in type, so each
-// lane tests admission with the masked XOR.
+// The wildcard chain in its leanest form, software-pipelined.  Lane l owns
+// tuple k (own) and keeps in registers cur = its exact receives posted before
+// the current wildcard (advanced with a cursor npos over the tuple's
+// posting-ordered receive positions) and c = the wildcards it served so far;
+// its candidate is list_k[cur + c].  Wildcards are served in posting order
+// from wl[x_begin..W) -- those with in(y) --, 32 positions at a time held in
+// registers; `left` of them in all.  While the redux.sync.min of step t is in
+// flight the warp already finds wildcard t + 1, advances cur to it and loads
+// list_k[cur + c] and list_k[cur + c + 1] -- the candidates for a loss and for
+// a win at step t --, so a step's critical path is the reduction and a select.
+// ADMIT: wildcards may differ in type, so each lane tests admission with the
+// masked XOR.
 template <bool ADMIT, class InF, class HdrF>
 __device__ __forceinline__ void lean_chain(const FifoWs& ws, bool own, uint32_t k, uint32_t x_begin, uint32_t W,
                                            uint32_t left, InF in_chain, HdrF hdrof, int lane) {
+  if (left == 0) return;
   uint32_t st = 0, hend = 0, rs = 0, rc = 0;
   uint64_t kh = 0;
   if (own) {
@@ -281,43 +284,66 @@ __device__ __forceinline__ void lean_chain(const FifoWs& ws, bool own, uint32_t 
     rc = ws.key_rcnt[k];
     if (ADMIT) kh = ws.keyhdr[k];
   }
-  uint32_t cur = 0, c = 0, hp = st;
+  uint32_t cur = 0, c = 0;
   uint32_t npos = rc ? (uint32_t)ws.rby_key[rs] : 0xFFFFFFFFu;
-  uint32_t h0 = hp < hend ? (uint32_t)ws.by_key[hp] : 0xFFFFFFFFu;
-  uint32_t h1 = hp + 1 < hend ? (uint32_t)ws.by_key[hp + 1] : 0xFFFFFFFFu;
-  for (uint32_t cb = x_begin & ~31u; left > 0; cb += 32) {
+  auto head = [&](uint32_t p) { return p < hend ? (uint32_t)ws.by_key[p] : 0xFFFFFFFFu; };
+  auto advance = [&](uint32_t w) {  // exact receives of k posted before w
+    while (npos < w) {
+      cur++;
+      npos = cur < rc ? (uint32_t)ws.rby_key[rs + cur] : 0xFFFFFFFFu;
+    }
+  };
+  // cursor over the chain's wildcards (warp-uniform)
+  uint32_t cb = x_begin & ~31u, cm = 0, wv = 0;
+  uint64_t rv = 0;
+  auto load_chunk = [&]() {
     const uint32_t y = cb + lane;
     const bool in = y >= x_begin && y < W && in_chain(y);
-    uint32_t cm = __ballot_sync(kFull, in);
-    const uint32_t wv = in ? (uint32_t)ws.wl[y] : 0u;
-    const uint64_t rv = (ADMIT && in) ? hdrof(y) : 0ull;
-    while (cm) {
-      const int bit = __ffs(cm) - 1;
-      cm &= cm - 1;
-      left--;
-      const uint32_t w = __shfl_sync(kFull, wv, bit);
-      while (npos < w) {  // exact receives of k posted before w take heads first
-        cur++;
-        npos = cur < rc ? (uint32_t)ws.rby_key[rs + cur] : 0xFFFFFFFFu;
-        hp++;
-        h0 = h1;
-        h1 = hp + 1 < hend ? (uint32_t)ws.by_key[hp + 1] : 0xFFFFFFFFu;
-      }
-      uint32_t cand = h0;
-      if (ADMIT) {
-        const uint64_t r = __shfl_sync(kFull, rv, bit);
-        if (((kh ^ r) & wildcard_mask(r)) != 0) cand = 0xFFFFFFFFu;
-      }
-      const uint32_t win = __reduce_min_sync(kFull, cand);
-      if (win != 0xFFFFFFFFu && cand == win) {
-        ws.wlog[st + c] = (uint16_t)w;
-        c++;
-        hp++;
-        h0 = h1;
-        h1 = hp + 1 < hend ? (uint32_t)ws.by_key[hp + 1] : 0xFFFFFFFFu;
-      }
-      if (lane == 0) ws.recv_res[cb + bit] = win == 0xFFFFFFFFu ? kNone : (uint16_t)win;
+    cm = __ballot_sync(kFull, in);
+    wv = in ? (uint32_t)ws.wl[y] : 0u;
+    if (ADMIT) rv = in ? hdrof(y) : 0ull;
+  };
+  auto next = [&](uint32_t& w, uint32_t& y, uint64_t& r) {
+    while (cm == 0) {
+      cb += 32;
+      load_chunk();
     }
+    const int bit = __ffs(cm) - 1;
+    cm &= cm - 1;
+    w = __shfl_sync(kFull, wv, bit);
+    y = cb + bit;
+    if (ADMIT) r = __shfl_sync(kFull, rv, bit);
+  };
+  load_chunk();
+  uint32_t w, y;
+  uint64_t r = 0;
+  next(w, y, r);
+  advance(w);
+  uint32_t cand = head(st + cur + c);
+  while (true) {
+    if (ADMIT && ((kh ^ r) & wildcard_mask(r)) != 0) cand = 0xFFFFFFFFu;
+    const uint32_t win = __reduce_min_sync(kFull, cand);
+    // lookahead, independent of this step's outcome
+    const bool more = --left > 0;
+    uint32_t w2 = 0, y2 = 0, l0 = 0xFFFFFFFFu, l1 = 0xFFFFFFFFu;
+    uint64_t r2 = 0;
+    if (more) {
+      next(w2, y2, r2);
+      advance(w2);
+      l0 = head(st + cur + c);
+      l1 = head(st + cur + c + 1);
+    }
+    const bool won = win != 0xFFFFFFFFu && cand == win;
+    if (won) {
+      ws.wlog[st + c] = (uint16_t)w;
+      c++;
+    }
+    if (lane == 0) ws.recv_res[y] = win == 0xFFFFFFFFu ? kNone : (uint16_t)win;
+    if (!more) break;
+    cand = won ? l1 : l0;
+    w = w2;
+    y = y2;
+    r = r2;
   }
   if (own) ws.key_c[k] = (uint16_t)c;
 }
