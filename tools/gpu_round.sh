@@ -12,8 +12,11 @@ print('clocks', d['clocks'])
 for k,v in d['levels'].items(): print(k, round(v['value']/1e9,3), 'Gm/s', round(v['ms_per_step'],3), 'ms kernel', round(v['roofline']['kernel_ms'],3), 'frac', round(v['roofline']['frac'],4))"
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv \
     --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline > gpurun_out/ncu_launch_$TAG.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_mpi_fifo|k_mpi_matrix" -s 6 -c 2 -o gpurun_out/prof_mpi_$TAG \
-    python bench.py --steps 1 --warmup 3 --levels mpi,mpi_matrix --no-cpu-baseline > gpurun_out/ncu_mpi_$TAG.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_part_scatter|k_bucket_pair|k_part_hist|k_bucket_bounds" -s 20 -c 8 -o gpurun_out/prof_flat_$TAG \
+# device-input launches only (the e2e leg's pipelined launches cover a quarter of the endpoints each)
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_mpi_fifo" -s 2 -c 1 -o gpurun_out/prof_mpi_$TAG \
+    python bench.py --steps 1 --warmup 3 --levels mpi --no-cpu-baseline > gpurun_out/ncu_mpi_$TAG.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_mpi_matrix" -s 2 -c 1 -o gpurun_out/prof_mpim_$TAG \
+    python bench.py --steps 1 --warmup 3 --levels mpi_matrix --no-cpu-baseline > gpurun_out/ncu_mpim_$TAG.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_part_scatter|k_bucket_pair|k_bucket_pop|k_part_hist|k_bucket_bounds" -s 20 -c 10 -o gpurun_out/prof_flat_$TAG \
     python bench.py --steps 1 --warmup 3 --levels ordered,unordered --no-cpu-baseline > gpurun_out/ncu_flat_$TAG.log 2>&1
 ls gpurun_out | grep $TAG

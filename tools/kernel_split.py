@@ -23,7 +23,7 @@ else:
     q = bench.ordered_workload(0, 1) if level == "ordered" else bench.unordered_workload(0)
     n = len(q.recv_hdr)
     sem = mm.MM_SEM_NOWILD_ORDERED if level == "ordered" else mm.MM_SEM_NOWILD_UNORDERED
-    eng = mm.Engine(sem, 1, n, n)
+    eng = mm.Engine(sem, 1, n, n, flat_kernel=int(os.environ.get("FLAT", "0")))
     rh, mh = bench.to_dev(q.recv_hdr), bench.to_dev(q.msg_hdr)
     def step():
         eng.reset(); eng.post_recvs(rh); eng.push_msgs(mh); eng.match_batch(orc, omc, cnt)
