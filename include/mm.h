@@ -222,7 +222,8 @@ enum { MM_MPI_KERNEL_AUTO = 0, MM_MPI_KERNEL_MATRIX = 1, MM_MPI_KERNEL_FIFO = 2 
 enum { MM_FLAT_KERNEL_BUCKETED = 0, MM_FLAT_KERNEL_GLOBAL = 1 };
 /*   MM_OPT_PIPELINE_CHUNKS: endpoint ranges of the MPI level's host-buffer
  *     pipeline (H2D of range k+1, matching of range k and D2H of range k-1
- *     overlap on three streams): 0 = auto (4 at >= 256 endpoints, else 1), 1 = off, 2..32 = that many ranges.  Results are identical
+ *     overlap on three streams): 0 = auto (6 at >= 1024 endpoints, 4 at >= 256, else 1;
+ *     ranges grow linearly towards the middle), 1 = off, 2..32 = that many ranges.  Results are identical
  *     for every value; a change applies to the next post. */
 int mm_set_option(mm_engine *e, int32_t option, int64_t value);
 

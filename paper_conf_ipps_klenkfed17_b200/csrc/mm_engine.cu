@@ -169,13 +169,24 @@ struct mm_engine {
   int pipeline = 0;          // MM_OPT_PIPELINE_CHUNKS (0 = auto)
 };
 
-static int64_t chunk_ep(const mm_engine* e, int k, int C) { return (int64_t)k * e->n_ep / C; }
+// Range k of C covers endpoints [chunk_ep(k), chunk_ep(k + 1)).  Ranges grow
+// linearly towards the middle (weights min(j + 1, C - j)): the first range's
+// copy-in and the last range's copy-out are the only transfers nothing
+// overlaps, so they are the smallest.
+static int64_t chunk_weight_sum(int k, int C) {
+  int64_t s = 0;
+  for (int j = 0; j < k; j++) s += (j + 1 < C - j) ? j + 1 : C - j;
+  return s;
+}
+static int64_t chunk_ep(const mm_engine* e, int k, int C) {
+  return (int64_t)e->n_ep * chunk_weight_sum(k, C) / chunk_weight_sum(C, C);
+}
 
 // Number of endpoint ranges the host-buffer pipeline uses (1 = no pipeline).
 static int pipeline_chunks(const mm_engine* e) {
   if (e->sem != MM_SEM_MPI || e->n_ep < 2) return 1;
   int C = e->pipeline;
-  if (C == 0) C = e->n_ep >= 256 ? 4 : 1;
+  if (C == 0) C = e->n_ep >= 1024 ? 6 : (e->n_ep >= 256 ? 4 : 1);
   return C < e->n_ep ? C : e->n_ep;
 }
 

@@ -44,7 +44,7 @@ def t_ms(fn, k=10):
     return a.elapsed_time(b) / k
 
 
-for c in [1, 2, 4, 8, 16, 32]:
+for c in [1, 2, 4, 6, 8, 12, 16, 24, 32]:
     eng.set_option(MM_OPT_PIPELINE_CHUNKS, c)
     print("chunks %2d  e2e %.3f ms/step" % (c, t_ms(step)))
 
@@ -74,10 +74,11 @@ bo = t_ms(both)
 print("H2D %.1f GB/s  D2H %.1f GB/s  (%d MB each)" % (nb / h2d / 1e6, nb / d2h / 1e6, nb >> 20))
 print("concurrent H2D+D2H of %d MB each: %.3f ms (%.1f GB/s per direction)" % (nb >> 21, bo, nb / 2 / bo / 1e6))
 
-eng.set_option(MM_OPT_PIPELINE_CHUNKS, 8)
+eng.set_option(MM_OPT_PIPELINE_CHUNKS, int(os.environ.get("TL_CHUNKS", "6")))
 step()
 torch.cuda.synchronize()
 with profile(activities=[ProfilerActivity.CUDA]) as prof:
+    step()
     step()
     torch.cuda.synchronize()
 evs = sorted([e for e in prof.events() if e.device_type == torch.autograd.DeviceType.CUDA],
