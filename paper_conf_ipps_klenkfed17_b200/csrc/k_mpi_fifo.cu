@@ -379,6 +379,14 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     const uint32_t mq1 = (nm + 3) / 4, mq2 = (2 * nm + 3) / 4, mq3 = (3 * nm + 3) / 4;
     const uint32_t rq1 = (nr + 3) / 4, rq2 = (2 * nr + 3) / 4, rq3 = (3 * nr + 3) / 4;
     MM_PHASE(0);
+    // the first round of message headers is requested before P1, so their
+    // HBM latency overlaps the table clearing and the barrier
+    uint64_t hv[4];
+#pragma unroll
+    for (int u = 0; u < 4; u++) {
+      const uint32_t j = tid + u * NT;
+      hv[u] = j < nm ? MS.hdr(j) : 0ull;
+    }
 
     // P1 -------------------------------------------------------------------
     for (uint32_t s = tid; s < H / 4; s += NT) reinterpret_cast<uint4*>(ws.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
@@ -398,11 +406,12 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     // insert message tuples; the CAS winner of a slot takes the next dense
     // tuple id and initialises the tuple's entries before publishing it
     for (uint32_t j0 = tid; j0 < nm; j0 += 4 * NT) {
-      uint64_t hv[4];
+      if (j0 != (uint32_t)tid) {
 #pragma unroll
-      for (int u = 0; u < 4; u++) {  // read once from HBM, four loads in flight
-        const uint32_t j = j0 + u * NT;
-        hv[u] = j < nm ? MS.hdr(j) : 0ull;
+        for (int u = 0; u < 4; u++) {  // read once from HBM, four loads in flight
+          const uint32_t j = j0 + u * NT;
+          hv[u] = j < nm ? MS.hdr(j) : 0ull;
+        }
       }
 #pragma unroll
       for (int u = 0; u < 4; u++) {
@@ -443,16 +452,23 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         inc16(&ws.pcnt[q * ws.mcap + id]);
       }
     }
+    // the first round of receive headers, requested before the barrier
+#pragma unroll
+    for (int u = 0; u < 4; u++) {
+      const uint32_t i = tid + u * NT;
+      hv[u] = i < nr ? RS.hdr(i) : 0ull;
+    }
     __syncthreads();
     MM_PHASE(2);
     const uint32_t K = sh_K;
     // P4 -------------------------------------------------------------------
     for (uint32_t i0 = tid; i0 < nr; i0 += 4 * NT) {
-      uint64_t hv[4];
+      if (i0 != (uint32_t)tid) {
 #pragma unroll
-      for (int u = 0; u < 4; u++) {  // four independent HBM loads in flight
-        const uint32_t i = i0 + u * NT;
-        hv[u] = i < nr ? RS.hdr(i) : 0ull;
+        for (int u = 0; u < 4; u++) {  // four independent HBM loads in flight
+          const uint32_t i = i0 + u * NT;
+          hv[u] = i < nr ? RS.hdr(i) : 0ull;
+        }
       }
 #pragma unroll
       for (int u = 0; u < 4; u++) {
