@@ -65,15 +65,34 @@ def load_peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def load_traffic(kernel):
-    """dram bytes per launch of `kernel` from the committed ncu capture summary."""
+def load_traffic(kernel, key="dram_bytes_per_launch"):
+    """Per-launch ncu counters of `kernel` from the committed capture summary
+    (profiles/kernel_traffic.json: dram bytes, warp instructions, issue %)."""
     p = os.path.join(ROOT, "profiles", "kernel_traffic.json")
     if not os.path.exists(p):
         return None
     with open(p) as f:
         d = json.load(f)
     v = d.get(kernel)
-    return v.get("dram_bytes_per_launch") if isinstance(v, dict) else None
+    return v.get(key) if isinstance(v, dict) else None
+
+
+def issue_efficiency(kernel, kernel_ms, sm_mhz):
+    """Warp-issue efficiency of `kernel` (north_star: "warp-issue efficiency"):
+    its warp instructions per launch (ncu capture) over the live kernel time,
+    against the issue peak of 4 warp instructions per SM per clock (one per
+    SM sub-partition) x SMs x the sampled SM clock; plus ncu's own
+    issue-active percentage of the captured launch."""
+    import torch
+    inst = load_traffic(kernel, "warp_inst_per_launch")
+    if not inst or not kernel_ms:
+        return None
+    sms = torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
+    peak = 4.0 * sms * sm_mhz * 1e6 / 1e9
+    ach = inst / (kernel_ms / 1e3) / 1e9
+    return {"kernel": kernel, "warp_inst_per_launch": inst, "achieved": ach, "peak": peak,
+            "unit": "G warp-inst/s", "frac": ach / peak, "sm_mhz": sm_mhz, "sms": sms,
+            "ncu_issue_active_pct": load_traffic(kernel, "issue_active_pct")}
 
 
 class Clocks:
@@ -411,6 +430,10 @@ def main():
             levels[lv] = bench_flat(args, world, rank, peak, lv)
     ck = clocks.stop()
     finalize_values(levels, args.steps)
+    for lv in levels.values():
+        rf = lv["roofline"]
+        if rf.get("kernel", "").startswith("k_mpi"):
+            lv["issue"] = issue_efficiency(rf["kernel"], rf.get("kernel_ms"), ck.get("sm_max_mhz") or 1965.0)
     head = levels.get("mpi") or next(iter(levels.values()))
     line = {
         "metric": METRIC, "value": head["value"], "unit": "matches/s", "n_gpus": world, "steps": args.steps,
@@ -420,6 +443,7 @@ def main():
                    "l2": "inputs > L2: 4 rotating copies of the configs[1] headers (256 MB); relaxed levels "
                          "use 256-512 MB inputs", "parallelism": "endpoints split over %d GPU(s)" % world},
         "roofline": {k: v for k, v in head["roofline"].items()},
+        "issue": head.get("issue"),
         "e2e": head.get("e2e"),
         "gpu_launches": head["_launches"],
         "clocks": ck,

@@ -99,15 +99,19 @@ def full(path, out, traffic=None):
             scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(u, 1)
             return x * scale
         b = num("dram__bytes_read.sum") + num("dram__bytes_write.sum")
-        d = tr.setdefault(short, {"launches": 0, "dram_bytes": 0.0})
+        d = tr.setdefault(short, {"launches": 0, "dram_bytes": 0.0, "inst": 0.0, "issue": 0.0})
         d["launches"] += 1
         d["dram_bytes"] += b
+        d["inst"] += num("smsp__inst_executed.sum")
+        d["issue"] += num("smsp__issue_active.avg.pct_of_peak_sustained_active")
     open(out, "w").write("\n".join(lines) + "\n")
     print("\n".join(lines[:60]))
     if traffic:
         old = json.load(open(traffic)) if __import__("os").path.exists(traffic) else {}
         for k, d in tr.items():
-            old[k] = {"dram_bytes_per_launch": d["dram_bytes"] / d["launches"], "source": path.split("/")[-1]}
+            n = d["launches"]
+            old[k] = {"dram_bytes_per_launch": d["dram_bytes"] / n, "warp_inst_per_launch": d["inst"] / n,
+                      "issue_active_pct": d["issue"] / n, "source": path.split("/")[-1]}
         json.dump(old, open(traffic, "w"), indent=1)
 
 
