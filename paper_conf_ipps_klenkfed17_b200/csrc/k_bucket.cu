@@ -588,10 +588,25 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cuda
   SnapRead rs{a.R.q_hdr, a.R.p_hdr, s.rres}, ms{a.M.q_hdr, a.M.p_hdr, s.mres};
   uint64_t *rh, *mh;
   uint64_t *ri, *mi;
-  cudaError_t err = partition_side(rs, a.nr, nb, s.h[0], s.i[0], s.h[1], s.i[1], s.part, s.roff, &rh, &ri, st);
+  // the two sides are independent until the bucket kernel: the messages are
+  // partitioned on a second stream (their small scan kernels and launch gaps
+  // overlap the receives' passes)
+  cudaStream_t mst = st;
+  cudaError_t err;
+  if (s.side_st) {
+    if ((err = cudaEventRecord(s.ev_fork, st)) != cudaSuccess) return err;
+    if ((err = cudaStreamWaitEvent(s.side_st, s.ev_fork, 0)) != cudaSuccess) return err;
+    mst = s.side_st;
+  }
+  err = partition_side(rs, a.nr, nb, s.h[0], s.i[0], s.h[1], s.i[1], s.part, s.roff, &rh, &ri, st);
   if (err != cudaSuccess) return err;
-  err = partition_side(ms, a.nm, nb, s.h[2], s.i[2], s.h[3], s.i[3], s.part, s.moff, &mh, &mi, st);
+  err = partition_side(ms, a.nm, nb, s.h[2], s.i[2], s.h[3], s.i[3], s.side_st ? s.part2 : s.part, s.moff, &mh, &mi,
+                       mst);
   if (err != cudaSuccess) return err;
+  if (s.side_st) {
+    if ((err = cudaEventRecord(s.ev_join, s.side_st)) != cudaSuccess) return err;
+    if ((err = cudaStreamWaitEvent(st, s.ev_join, 0)) != cudaSuccess) return err;
+  }
   if ((err = cudaMemsetAsync(s.overflow, 0, 4, st)) != cudaSuccess) return err;
   s.rh_sorted = rh;
   s.ri_sorted = ri;

@@ -157,7 +157,9 @@ struct mm_engine {
   DBuf skey[2], sval[2], rid, run_start, run_rc, part;
   DBuf owner, rcnt, mcnt, tkey, tval;
   int64_t T = 0;
-  DBuf bh[4], bi[4], bpart, broff, bmoff, bover;
+  DBuf bh[4], bi[4], bpart, bpart2, broff, bmoff, bover;
+  cudaStream_t fs = nullptr;  // no-wildcard levels: the message side's partition stream
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   int flat_kernel = MM_FLAT_KERNEL_BUCKETED;
   long long bucket_fallbacks = 0;
   Timer timer;
@@ -261,6 +263,10 @@ int mm_destroy(mm_engine* e) {
       if (q->ev[k]) cudaEventDestroy(q->ev[k]);
   }
   if (e->ev_st) cudaEventDestroy(e->ev_st);
+  if (e->fs) cudaStreamSynchronize(e->fs);
+  if (e->fs) cudaStreamDestroy(e->fs);
+  if (e->ev_fork) cudaEventDestroy(e->ev_fork);
+  if (e->ev_join) cudaEventDestroy(e->ev_join);
   if (e->cs) cudaStreamDestroy(e->cs);
   if (e->ds) cudaStreamDestroy(e->ds);
   if (e->h_off) cudaFreeHost(e->h_off);
@@ -279,7 +285,7 @@ int mm_destroy(mm_engine* e) {
                   &e->sval[0], &e->sval[1], &e->rid, &e->run_start, &e->run_rc, &e->part,
                   &e->owner, &e->rcnt, &e->mcnt, &e->tkey, &e->tval, &e->fifo_ws,
                   &e->bh[0], &e->bh[1], &e->bh[2], &e->bh[3], &e->bi[0], &e->bi[1], &e->bi[2], &e->bi[3],
-                  &e->bpart, &e->broff, &e->bmoff, &e->bover};
+                  &e->bpart, &e->bpart2, &e->broff, &e->bmoff, &e->bover};
   for (DBuf* b : bufs) release(*b);
   delete e;
   return MM_OK;
@@ -341,7 +347,11 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
       const int64_t c = b < 2 ? e->rcap : e->mcap;
       ok = ensure(e->bh[b], c * 8) == cudaSuccess && ensure(e->bi[b], c * 8) == cudaSuccess;
     }
-    ok = ok && ensure(e->bpart, (size_t)partition_scratch_elems(e->rcap > e->mcap ? e->rcap : e->mcap) * 4) == cudaSuccess &&
+    ok = ok && ensure(e->bpart, (size_t)partition_scratch_elems(e->rcap) * 4) == cudaSuccess &&
+         ensure(e->bpart2, (size_t)partition_scratch_elems(e->mcap) * 4) == cudaSuccess &&
+         cudaStreamCreateWithFlags(&e->fs, cudaStreamNonBlocking) == cudaSuccess &&
+         cudaEventCreateWithFlags(&e->ev_fork, cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming) == cudaSuccess &&
          ensure(e->broff, (size_t)bucket_scratch_elems(n) * 4) == cudaSuccess &&
          ensure(e->bmoff, (size_t)bucket_scratch_elems(n) * 4) == cudaSuccess && ensure(e->bover, 4) == cudaSuccess;
     if (ok && semantics == MM_SEM_NOWILD_ORDERED) {
@@ -669,6 +679,10 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
       bs.i[b] = (uint64_t*)e->bi[b].p;
     }
     bs.part = (uint32_t*)e->bpart.p;
+    bs.part2 = (uint32_t*)e->bpart2.p;
+    bs.side_st = e->fs;
+    bs.ev_fork = e->ev_fork;
+    bs.ev_join = e->ev_join;
     bs.roff = (uint32_t*)e->broff.p;
     bs.moff = (uint32_t*)e->bmoff.p;
     bs.overflow = (uint32_t*)e->bover.p;

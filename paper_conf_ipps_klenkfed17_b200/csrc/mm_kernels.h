@@ -96,10 +96,13 @@ cudaError_t run_hash(const FlatArgs& a, const HashScratch& h, cudaStream_t st);
 struct BucketScratch {
   uint64_t* h[4];  // receive ping-pong (0,1), message ping-pong (2,3)
   uint64_t* i[4];  // (bucket << 32) | snapshot index
-  uint32_t* part;
+  uint32_t* part;   // partition scratch of the receive side
+  uint32_t* part2;  // ... of the message side (partitioned concurrently on side_st)
   uint32_t* roff;
   uint32_t* moff;
   uint32_t* overflow;
+  cudaStream_t side_st;            // nullptr: both sides on the engine stream
+  cudaEvent_t ev_fork, ev_join;
   int64_t rres, mres;
   // outputs: the bucket-sorted sides (results are written in this order)
   const uint64_t* rh_sorted;

@@ -126,6 +126,42 @@ def test_mpi_host_pipeline_truncated_output():
     assert np.array_equal(g[0][0][:fit], o[0][0][:fit]) and np.array_equal(g[0][1][:fit], o[0][1][:fit])
 
 
+@pytest.mark.parametrize("chunks", [3, 6])
+def test_mpi_host_pipeline_two_posts_and_reset(chunks):
+    """Deferred host inputs: a second post before the match moves the first
+    (its chunk copies are issued and joined first); a reset drops a deferred
+    post without copying it; host outputs come back per range."""
+    rng = np.random.default_rng(5)
+    q = synth.mpi_endpoints(15, n_ep=300, depth_r=40, n_src=5, n_tag=3, p_any_src=0.3, p_any_tag=0.2,
+                            ragged=True, p_unmatched=0.2)
+    b1, b2 = split_batches(q, 2, rng)
+    from paper_conf_ipps_klenkfed17_b200 import Engine
+    from paper_conf_ipps_klenkfed17_b200._lib import MM_OPT_PIPELINE_CHUNKS
+    eng = Engine(MPI, q.n_endpoints, 80, 80)
+    eng.set_option(MM_OPT_PIPELINE_CHUNKS, chunks)
+    junk = synth.mpi_endpoints(99, n_ep=300, depth_r=40, ragged=True)
+    eng.post_recvs(junk.recv_hdr.astype(np.uint64), None, junk.recv_off)  # dropped by the reset
+    eng.reset()
+    for (rh, rc, ro, mh, mc, mo) in (b1, b2):  # both halves posted before one match
+        eng.post_recvs(np.ascontiguousarray(rh, np.uint64), rc, ro)
+        eng.push_msgs(np.ascontiguousarray(mh, np.uint64), mc, mo)
+    cap = q.n_endpoints * 80
+    orc = np.full(cap, -7, np.int64)
+    omc = np.full(cap, -7, np.int64)
+    cnt = np.zeros(2, np.int64)
+    eng.match_batch(orc, omc, cnt)
+    qs = eng.query()
+    eng.close()
+    oe = oracle.OracleEngine(MPI, q.n_endpoints)
+    for (rh, rc, ro, mh, mc, mo) in (b1, b2):
+        oe.post_recvs(rh, rc, ro)
+        oe.push_msgs(mh, mc, mo)
+    o_rc, o_mc = oe.match_batch()
+    n = int(cnt[0])
+    assert n == len(o_rc) and qs["error"] == 0
+    assert np.array_equal(orc[:n], o_rc) and np.array_equal(omc[:n], o_mc)
+
+
 @KERNELS
 def test_mpi_user_cookies_and_two_posts(kern):
     """Cookies are carried through; a second post before a match is queued."""
