@@ -442,121 +442,138 @@ struct PopSmem {
   uint32_t matched[kBucketCap / 32];      // message matched bits (by message offset)
 };
 
-__global__ void __launch_bounds__(kBucketThreads) k_bucket_pop(BucketArgs ba) {
+__global__ void __launch_bounds__(kBucketThreads) k_bucket_pop(BucketArgs ba, uint32_t nbk) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   PopSmem& sm = *reinterpret_cast<PopSmem*>(smem_raw);
   constexpr int NT = kBucketThreads;
+  constexpr int PER = kBucketCap / NT;
   const int tid = threadIdx.x, lane = tid & 31;
   const FlatArgs& a = ba.a;
-  const int b = blockIdx.x;
-  const uint32_t r0 = ba.roff[b], nr = ba.roff[b + 1] - r0;
-  const uint32_t m0 = ba.moff[b], nm = ba.moff[b + 1] - m0;
-  if (nr + nm == 0) return;
-  if (nr + nm > (uint32_t)kBucketCap) {
-    if (tid == 0) atomicOr(ba.overflow, 1u);
-    return;
-  }
-  const uint32_t n = nr + nm;
   const int64_t rres = a.R.q_len[0], rpb = a.R.pend_begin(0);
   const int64_t mres = a.M.q_len[0], mpb = a.M.pend_begin(0);
   constexpr uint32_t hmask = kBucketH - 1;
-  // load (all loads of a thread in flight), clear the tables
-  {
-    constexpr int PER = kBucketCap / NT;
-    uint64_t hv[PER], iv[PER];
+  // Persistent: buckets blockIdx.x, + gridDim.x, ...; the next bucket's
+  // elements are loaded into registers while the current one is matched.
+  uint64_t hv[PER];
+  uint32_t iv[PER];
+  auto fetch = [&](uint32_t bb, uint32_t& fr0, uint32_t& fnr, uint32_t& fm0, uint32_t& fnm) {
+    fr0 = fnr = fm0 = fnm = 0;
+    if (bb < nbk) {
+      fr0 = ba.roff[bb];
+      fnr = ba.roff[bb + 1] - fr0;
+      fm0 = ba.moff[bb];
+      fnm = ba.moff[bb + 1] - fm0;
+    }
+    const bool fits = fnr + fnm <= (uint32_t)kBucketCap;
 #pragma unroll
     for (int u = 0; u < PER; u++) {
       const uint32_t e = tid + u * NT;
       hv[u] = 0;
       iv[u] = 0;
-      if (e < nr) {
-        hv[u] = ba.rh[r0 + e];
-        iv[u] = ba.ri[r0 + e];
-      } else if (e < n) {
-        hv[u] = ba.mh[m0 + e - nr];
-        iv[u] = ba.mi[m0 + e - nr];
+      if (fits && e < fnr) {
+        hv[u] = ba.rh[fr0 + e];
+        iv[u] = (uint32_t)ba.ri[fr0 + e];
+      } else if (fits && e < fnr + fnm) {
+        hv[u] = ba.mh[fm0 + e - fnr];
+        iv[u] = (uint32_t)ba.mi[fm0 + e - fnr];
       }
     }
-    for (uint32_t s = tid; s < kBucketH / 4; s += NT) reinterpret_cast<uint4*>(sm.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
-    for (uint32_t s = tid; s < kBucketH / 8; s += NT) reinterpret_cast<uint4*>(sm.mhead)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
-    for (uint32_t s = tid; s < kBucketCap / 32; s += NT) sm.matched[s] = 0u;
+  };
+  uint32_t xr0, xnr, xm0, xnm;  // bounds of the bucket held in hv / iv
+  fetch(blockIdx.x, xr0, xnr, xm0, xnm);
+  for (uint32_t b = blockIdx.x; b < nbk; b += gridDim.x) {
+    __syncthreads();  // the previous bucket is done with shared memory
+    const uint32_t r0 = xr0, nr = xnr, m0 = xm0, nm = xnm;
+    const uint32_t n = nr + nm;
+    if (n == 0 || n > (uint32_t)kBucketCap) {  // uniform across the CTA
+      if (n > (uint32_t)kBucketCap && tid == 0) atomicOr(ba.overflow, 1u);
+      fetch(b + gridDim.x, xr0, xnr, xm0, xnm);
+      continue;
+    }
+    // registers to shared memory, clear the tables, prefetch the next bucket
+    {
 #pragma unroll
-    for (int u = 0; u < PER; u++) {
-      const uint32_t e = tid + u * NT;
-      if (e < n) {
-        sm.hdr[e] = hv[u];
-        sm.idx[e] = (uint32_t)iv[u];
+      for (int u = 0; u < PER; u++) {
+        const uint32_t e = tid + u * NT;
+        if (e < n) {
+          sm.hdr[e] = hv[u];
+          sm.idx[e] = iv[u];
+        }
       }
+      for (uint32_t s = tid; s < kBucketH / 4; s += NT) reinterpret_cast<uint4*>(sm.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
+      for (uint32_t s = tid; s < kBucketH / 8; s += NT) reinterpret_cast<uint4*>(sm.mhead)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
+      for (uint32_t s = tid; s < kBucketCap / 32; s += NT) sm.matched[s] = 0u;
+      fetch(b + gridDim.x, xr0, xnr, xm0, xnm);
     }
-  }
-  __syncthreads();
-  // messages: find or open the tuple's slot, push onto its message list
-  for (uint32_t e = nr + tid; e < n; e += NT) {
-    const uint64_t h = sm.hdr[e];
-    const uint64_t p = h * 0xD6E8FEB86659FD93ull;
-    uint32_t s = (uint32_t)(p >> 40) & hmask;
-    const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
-    while (true) {
-      uint32_t o = sm.table[s];
-      if (o == 0xFFFFFFFFu) {
-        o = atomicCAS(&sm.table[s], 0xFFFFFFFFu, (fp << 16) | e);  // representative's header is in smem already
+    __syncthreads();
+    // messages: find or open the tuple's slot, push onto its message list
+    for (uint32_t e = nr + tid; e < n; e += NT) {
+      const uint64_t h = sm.hdr[e];
+      const uint64_t p = h * 0xD6E8FEB86659FD93ull;
+      uint32_t s = (uint32_t)(p >> 40) & hmask;
+      const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
+      while (true) {
+        uint32_t o = sm.table[s];
+        if (o == 0xFFFFFFFFu) {
+          o = atomicCAS(&sm.table[s], 0xFFFFFFFFu, (fp << 16) | e);  // representative's header is in smem already
+          if (o == 0xFFFFFFFFu) break;
+        }
+        if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) break;
+        s = (s + 1) & hmask;
+      }
+      sm.next[e] = exch16(&sm.mhead[s], (uint16_t)e);
+    }
+    __syncthreads();
+    // receives: look the tuple up
+    for (uint32_t e = tid; e < nr; e += NT) {
+      const uint64_t h = sm.hdr[e];
+      const uint64_t p = h * 0xD6E8FEB86659FD93ull;
+      uint32_t s = (uint32_t)(p >> 40) & hmask;
+      const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
+      uint32_t found = kNone;
+      while (true) {
+        const uint32_t o = sm.table[s];
         if (o == 0xFFFFFFFFu) break;
-      }
-      if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) break;
-      s = (s + 1) & hmask;
-    }
-    sm.next[e] = exch16(&sm.mhead[s], (uint16_t)e);
-  }
-  __syncthreads();
-  // receives: look the tuple up
-  for (uint32_t e = tid; e < nr; e += NT) {
-    const uint64_t h = sm.hdr[e];
-    const uint64_t p = h * 0xD6E8FEB86659FD93ull;
-    uint32_t s = (uint32_t)(p >> 40) & hmask;
-    const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
-    uint32_t found = kNone;
-    while (true) {
-      const uint32_t o = sm.table[s];
-      if (o == 0xFFFFFFFFu) break;
-      if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) {
-        found = s;
-        break;
-      }
-      s = (s + 1) & hmask;
-    }
-    sm.slot[e] = (uint16_t)found;
-  }
-  __syncthreads();
-  // receives take any message of their tuple (pop from the list)
-  uint32_t nmatch = 0;
-  for (uint32_t e = tid; e < nr; e += NT) {
-    const uint32_t s = sm.slot[e];
-    uint32_t j = kNone;
-    if (s != kNone) {
-      uint32_t hd = sm.mhead[s];
-      while (hd != kNone) {  // pops only in this phase: no ABA
-        const uint32_t got = cas16(&sm.mhead[s], (uint16_t)hd, sm.next[hd]);
-        if (got == hd) {
-          j = hd;
+        if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) {
+          found = s;
           break;
         }
-        hd = got;
+        s = (s + 1) & hmask;
       }
+      sm.slot[e] = (uint16_t)found;
     }
-    int64_t mc = MM_NO_MATCH;
-    if (j != kNone) {
-      atomicOr(&sm.matched[(j - nr) >> 5], 1u << ((j - nr) & 31));
-      mc = a.M.cookie(0, sm.idx[j], mres, mpb);
-      nmatch++;
+    __syncthreads();
+    // receives take any message of their tuple (pop from the list)
+    uint32_t nmatch = 0;
+    for (uint32_t e = tid; e < nr; e += NT) {
+      const uint32_t s = sm.slot[e];
+      uint32_t j = kNone;
+      if (s != kNone) {
+        uint32_t hd = sm.mhead[s];
+        while (hd != kNone) {  // pops only in this phase: no ABA
+          const uint32_t got = cas16(&sm.mhead[s], (uint16_t)hd, sm.next[hd]);
+          if (got == hd) {
+            j = hd;
+            break;
+          }
+          hd = got;
+        }
+      }
+      int64_t mc = MM_NO_MATCH;
+      if (j != kNone) {
+        atomicOr(&sm.matched[(j - nr) >> 5], 1u << ((j - nr) & 31));
+        mc = a.M.cookie(0, sm.idx[j], mres, mpb);
+        nmatch++;
+      }
+      a.out_rc[r0 + e] = a.R.cookie(0, sm.idx[e], rres, rpb);
+      a.out_mc[r0 + e] = mc;
+      a.rflag[r0 + e] = j != kNone ? 1 : 0;
     }
-    a.out_rc[r0 + e] = a.R.cookie(0, sm.idx[e], rres, rpb);
-    a.out_mc[r0 + e] = mc;
-    a.rflag[r0 + e] = j != kNone ? 1 : 0;
+    for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
+    if (lane == 0 && nmatch) atomicAdd(a.n_matched, (unsigned long long)nmatch);
+    __syncthreads();
+    for (uint32_t x = tid; x < nm; x += NT) a.mflag[m0 + x] = (sm.matched[x >> 5] >> (x & 31)) & 1u;
   }
-  for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
-  if (lane == 0 && nmatch) atomicAdd(a.n_matched, (unsigned long long)nmatch);
-  __syncthreads();
-  for (uint32_t x = tid; x < nm; x += NT) a.mflag[m0 + x] = (sm.matched[x >> 5] >> (x & 31)) & 1u;
 }
 
 // ~512 elements per bucket on average (capacity 1024: a bucket overflows
@@ -624,7 +641,7 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cuda
     err = cudaFuncSetAttribute(k_bucket_pop, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (err != cudaSuccess) return err;
     count_launch();
-    k_bucket_pop<<<B, kBucketThreads, smem, st>>>(ba);
+    k_bucket_pop<<<bucket_grid(k_bucket_pop, kBucketThreads, smem, B), kBucketThreads, smem, st>>>(ba, B);
   }
   return cudaGetLastError();
 }
