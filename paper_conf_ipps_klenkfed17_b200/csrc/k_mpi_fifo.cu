@@ -285,12 +285,18 @@ __device__ __forceinline__ void lean_chain(const FifoWs& ws, bool own, uint32_t 
     if (ADMIT) kh = ws.keyhdr[k];
   }
   uint32_t cur = 0, c = 0;
-  uint32_t npos = rc ? (uint32_t)ws.rby_key[rs] : 0xFFFFFFFFu;
+  // the next four exact-receive positions of k in registers: the cursor
+  // advances without waiting on a shared-memory load per step
+  auto rpos = [&](uint32_t x) { return x < rc ? (uint32_t)ws.rby_key[rs + x] : 0xFFFFFFFFu; };
+  uint32_t np0 = rpos(0), np1 = rpos(1), np2 = rpos(2), np3 = rpos(3);
   auto head = [&](uint32_t p) { return p < hend ? (uint32_t)ws.by_key[p] : 0xFFFFFFFFu; };
   auto advance = [&](uint32_t w) {  // exact receives of k posted before w
-    while (npos < w) {
+    while (np0 < w) {
       cur++;
-      npos = cur < rc ? (uint32_t)ws.rby_key[rs + cur] : 0xFFFFFFFFu;
+      np0 = np1;
+      np1 = np2;
+      np2 = np3;
+      np3 = rpos(cur + 3);
     }
   };
   // cursor over the chain's wildcards (warp-uniform)
@@ -347,6 +353,13 @@ __device__ __forceinline__ void lean_chain(const FifoWs& ws, bool own, uint32_t 
   }
   if (own) ws.key_c[k] = (uint16_t)c;
 }
+
+// wildcards of one type use the group chains above this many tuples (below,
+// one warp walks the receive queue: stream_chain)
+#ifndef MM_GROUP_MIN_K
+#define MM_GROUP_MIN_K 32
+#endif
+constexpr uint32_t kGroupMinK = MM_GROUP_MIN_K;
 
 template <int NT, bool SMEM>
 __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_t* gws) {
@@ -503,7 +516,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     }
     __syncthreads();
     const uint32_t types = sh_types;
-    const bool grouped = K > 32 && __popc(types) == 1;
+    const bool grouped = __popc(types) == 1 && K > kGroupMinK;
     MM_PHASE(4);
     // P5 -------------------------------------------------------------------
     uint32_t W;
@@ -595,7 +608,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     // higher warp ids first, so the critical path is not starved by the
     // parallel phases of co-resident CTAs (B300_MICROARCH.md, arbiter)
     if (W > 0) {
-      if (K <= 32) {
+      if (!grouped && K <= 32) {
         if (warp == NW - 1) stream_chain(ws, ws.gnext, nr, K, W, hdrof, lane);  // gnext is free here
         MM_PHASE(11);
 #ifdef MM_PHASE_TIMING
