@@ -19,4 +19,6 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_m
     python bench.py --steps 1 --warmup 3 --levels mpi_matrix --no-cpu-baseline > gpurun_out/ncu_mpim_$TAG.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_part_scatter|k_bucket_pair|k_bucket_pop|k_part_hist|k_bucket_bounds" -s 20 -c 10 -o gpurun_out/prof_flat_$TAG \
     python bench.py --steps 1 --warmup 3 --levels ordered,unordered --no-cpu-baseline > gpurun_out/ncu_flat_$TAG.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_bucket_pop" -s 2 -c 1 -o gpurun_out/prof_pop_$TAG \
+    python bench.py --steps 1 --warmup 3 --levels unordered --no-cpu-baseline > gpurun_out/ncu_pop_$TAG.log 2>&1
 ls gpurun_out | grep $TAG
