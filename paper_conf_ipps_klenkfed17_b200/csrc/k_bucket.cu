@@ -429,6 +429,9 @@ __global__ void __launch_bounds__(kPairThreads, 5) k_bucket_pair(BucketArgs ba, 
   }
 }
 
+#ifndef MM_POP_MIN_BLOCKS
+#define MM_POP_MIN_BLOCKS 6  // resident CTAs per SM the register budget must allow (28.8 KB smem allows 7)
+#endif
 // NOWILD_UNORDERED: messages pushed onto per-tuple lists, receives pop from
 // them (lock-free, pops only in that phase: no ABA) -- any maximal pairing of
 // equal tuples; 3 barriers.
@@ -442,7 +445,7 @@ struct PopSmem {
   uint32_t matched[kBucketCap / 32];      // message matched bits (by message offset)
 };
 
-__global__ void __launch_bounds__(kBucketThreads) k_bucket_pop(BucketArgs ba, uint32_t nbk) {
+__global__ void __launch_bounds__(kBucketThreads, MM_POP_MIN_BLOCKS) k_bucket_pop(BucketArgs ba, uint32_t nbk) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   PopSmem& sm = *reinterpret_cast<PopSmem*>(smem_raw);
   constexpr int NT = kBucketThreads;
