@@ -672,6 +672,7 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
   a.rflag = (uint8_t*)e->rflag.p;
   a.mflag = (uint8_t*)e->mflag.p;
   bool done = false;
+  unsigned long long matched_host = 0;  // pairs of the bucketed run (valid when done)
   BucketScratch bs;
   if (e->flat_kernel == MM_FLAT_KERNEL_BUCKETED) {
     for (int b = 0; b < 4; b++) {
@@ -693,6 +694,7 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
     e->timer.end(e->st);
     uint32_t over = 0;
     CK(cudaMemcpyAsync(&over, e->bover.p, 4, cudaMemcpyDeviceToHost, e->st));
+    CK(cudaMemcpyAsync(&matched_host, e->nmatched.p, 8, cudaMemcpyDeviceToHost, e->st));
     CK(cudaStreamSynchronize(e->st));
     done = over == 0;
     if (!done) {  // a bucket exceeded the on-chip capacity (heavily repeated tuples)
@@ -741,7 +743,11 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
   for (int i = 0; i < 2; i++) {
     Queue& q = *qs[i];
     const int nb = q.cur ^ 1;
-    if (done)  // bucketed: flags and survivors in bucket order
+    if (done && (int64_t)matched_host == ns[i]) {
+      // every element of this side matched (known from the count read back
+      // with the overflow flag): the residual queue is empty, no compaction
+      CK(cudaMemsetAsync(q.len[nb].p, 0, 4, e->st));
+    } else if (done)  // bucketed: flags and survivors in bucket order
       CK(run_compact_sorted(*ss[i], res[i], ns[i], i == 0 ? bs.rh_sorted : bs.mh_sorted,
                             i == 0 ? bs.ri_sorted : bs.mi_sorted, fl[i], (uint64_t*)q.hdr[nb].p,
                             (int64_t*)q.cookie[nb].p, (int32_t*)q.len[nb].p, (uint32_t*)e->scan.p, e->st));
@@ -750,8 +756,13 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
                      (int32_t*)q.len[nb].p, (uint32_t*)e->scan.p, e->st));
     q.cur = nb;
     q.pend = Pending();
-    q.resid_host = ns[i];  // upper bound until the next exact read
-    q.resid_exact = false;
+    if (done) {  // each pair consumed one element of each side: the residual size is exact
+      q.resid_host = ns[i] - (int64_t)matched_host;
+      q.resid_exact = true;
+    } else {
+      q.resid_host = ns[i];  // upper bound until the next exact read
+      q.resid_exact = false;
+    }
   }
   CK(launch_finalize(nullptr, nr, (const unsigned long long*)e->nmatched.p, (int64_t*)e->counts_dev.p, e->st));
   if (counts && !counts_host) CK(cudaMemcpyAsync(counts, e->counts_dev.p, 16, cudaMemcpyDeviceToDevice, e->st));
