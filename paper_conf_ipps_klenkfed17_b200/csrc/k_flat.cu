@@ -378,15 +378,38 @@ cudaError_t launch_materialize(const Side& S, int n_ep, uint64_t* q_h, int64_t* 
 }
 
 // ------------------------------------------------------------------ finalize
+// mm_reset: both queues' current lengths and the error flags in one launch
+__global__ void k_reset(int32_t* rlen, int32_t* mlen, int n_ep, uint32_t* err) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n_ep; i += gridDim.x * blockDim.x) {
+    rlen[i] = 0;
+    mlen[i] = 0;
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) *err = 0u;
+}
+cudaError_t launch_reset(int32_t* rlen, int32_t* mlen, int n_ep, uint32_t* err, cudaStream_t st) {
+  count_launch();
+  int grid = (n_ep + 255) / 256;
+  if (grid > 148 * 4) grid = 148 * 4;
+  k_reset<<<grid < 1 ? 1 : grid, 256, 0, st>>>(rlen, mlen, n_ep, err);
+  return cudaGetLastError();
+}
+
+// {n_out, n_matched} into the engine's counts and, if given, the caller's
+// device counts (one launch instead of a kernel and a copy)
 __global__ void k_finalize(const int64_t* n_out_src, int64_t n_out_host, const unsigned long long* n_matched,
-                           int64_t* counts) {
-  counts[0] = n_out_src ? *n_out_src : n_out_host;
-  counts[1] = (int64_t)*n_matched;
+                           int64_t* counts, int64_t* user_counts) {
+  const int64_t a = n_out_src ? *n_out_src : n_out_host, b = (int64_t)*n_matched;
+  counts[0] = a;
+  counts[1] = b;
+  if (user_counts) {
+    user_counts[0] = a;
+    user_counts[1] = b;
+  }
 }
 cudaError_t launch_finalize(const int64_t* n_out_src, int64_t n_out_host, const unsigned long long* n_matched,
-                            int64_t* counts, cudaStream_t st) {
+                            int64_t* counts, int64_t* user_counts, cudaStream_t st) {
   count_launch();
-  k_finalize<<<1, 1, 0, st>>>(n_out_src, n_out_host, n_matched, counts);
+  k_finalize<<<1, 1, 0, st>>>(n_out_src, n_out_host, n_matched, counts, user_counts);
   return cudaGetLastError();
 }
 

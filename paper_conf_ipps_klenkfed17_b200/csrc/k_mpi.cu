@@ -20,20 +20,26 @@
 
 namespace mm {
 
-__global__ void k_out_offsets(Side R, int n_ep, int64_t* out_off, int64_t out_cap, uint32_t* err) {
+// out_off[e] = first output slot of endpoint e (exclusive scan of the
+// snapshot receive counts); one CTA, each thread a contiguous run of
+// endpoints, one block scan.  Also zeroes the batch's pair counter.
+__global__ void k_out_offsets(Side R, int n_ep, int64_t* out_off, int64_t out_cap, uint32_t* err,
+                              unsigned long long* n_matched) {
   __shared__ int64_t sm[1024 / 32 + 1];
-  int64_t carry = 0;
-  for (int64_t b = 0; b < n_ep; b += blockDim.x) {
-    int64_t e = b + threadIdx.x;
-    int64_t v = e < n_ep ? (int64_t)R.q_len[e] + R.pend_count((int)e) : 0;
-    int64_t tot;
-    int64_t ex = block_excl_scan(v, sm, &tot);
-    if (e < n_ep) out_off[e] = carry + ex;
-    carry += tot;
+  const int per = (n_ep + (int)blockDim.x - 1) / (int)blockDim.x;
+  const int e0 = min(n_ep, (int)threadIdx.x * per), e1 = min(n_ep, e0 + per);
+  int64_t v = 0;
+  for (int e = e0; e < e1; e++) v += (int64_t)R.q_len[e] + R.pend_count(e);
+  int64_t tot;
+  int64_t run = block_excl_scan(v, sm, &tot);
+  for (int e = e0; e < e1; e++) {
+    out_off[e] = run;
+    run += (int64_t)R.q_len[e] + R.pend_count(e);
   }
   if (threadIdx.x == 0) {
-    out_off[n_ep] = carry;
-    if (carry > out_cap) atomicOr(err, kErrOutput);
+    out_off[n_ep] = tot;
+    if (tot > out_cap) atomicOr(err, kErrOutput);
+    if (n_matched) *n_matched = 0ull;
   }
 }
 
@@ -192,9 +198,9 @@ cudaError_t launch_mpi_matrix(const MpiArgs& a, cudaStream_t st) {
 }
 
 cudaError_t launch_out_offsets(const Side& R, int n_ep, int64_t* out_off, int64_t out_cap, uint32_t* err,
-                               cudaStream_t st) {
+                               unsigned long long* n_matched, cudaStream_t st) {
   count_launch();
-  k_out_offsets<<<1, 1024, 0, st>>>(R, n_ep, out_off, out_cap, err);
+  k_out_offsets<<<1, 1024, 0, st>>>(R, n_ep, out_off, out_cap, err, n_matched);
   return cudaGetLastError();
 }
 

@@ -512,17 +512,17 @@ int mm_push_msgs(mm_engine* e, const uint64_t* hdr, const int64_t* cookie, const
 
 int mm_reset(mm_engine* e) {
   if (!e) return MM_ERR_ARG;
+  LaunchScope ls(e);
+  // only the current ping-pong buffer (cur = 0) is read before it is written
+  CK(launch_reset((int32_t*)e->rq.len[0].p, (int32_t*)e->mq.len[0].p, e->n_ep, (uint32_t*)e->err.p, e->st));
   Queue* qs[2] = {&e->rq, &e->mq};
   for (Queue* q : qs) {
-    for (int b = 0; b < 2; b++)
-      if (q->len[b].p) CK(cudaMemsetAsync(q->len[b].p, 0, (size_t)e->n_ep * 4, e->st));
     q->pend = Pending();
     q->seq = 0;
     q->cur = 0;
     q->resid_host = 0;
     q->resid_exact = true;
   }
-  CK(cudaMemsetAsync(e->err.p, 0, 4, e->st));
   return MM_OK;
 }
 
@@ -568,8 +568,8 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
       if (jr != MM_OK) return jr;
     }
   Side R = make_side(e, e->rq, e->rcap), M = make_side(e, e->mq, e->mcap);
-  CK(cudaMemsetAsync(e->nmatched.p, 0, 8, e->st));
-  CK(launch_out_offsets(R, e->n_ep, (int64_t*)e->out_off.p, out_cap, (uint32_t*)e->err.p, e->st));
+  CK(launch_out_offsets(R, e->n_ep, (int64_t*)e->out_off.p, out_cap, (uint32_t*)e->err.p,
+                        (unsigned long long*)e->nmatched.p, e->st));  // also zeroes the pair counter
   if (host_out) {  // the output ranges are only known on the device: fetch them first
     CK(cudaMemcpyAsync(e->h_off, e->out_off.p, (size_t)(e->n_ep + 1) * 8, cudaMemcpyDeviceToHost, e->st));
     CK(cudaStreamSynchronize(e->st));
@@ -617,10 +617,9 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
   }
   e->timer.end(e->st);
   CK(launch_finalize((const int64_t*)e->out_off.p + e->n_ep, 0, (const unsigned long long*)e->nmatched.p,
-                     (int64_t*)e->counts_dev.p, e->st));
+                     (int64_t*)e->counts_dev.p, counts && !counts_host ? counts : nullptr, e->st));
   e->rq.pend = Pending();
   e->mq.pend = Pending();
-  if (counts && !counts_host) CK(cudaMemcpyAsync(counts, e->counts_dev.p, 16, cudaMemcpyDeviceToDevice, e->st));
   if (pipe) CK(cudaStreamSynchronize(e->cs));  // the caller may reuse its host inputs once we return
   if (pipe && host_out) {
     CK(cudaStreamSynchronize(e->ds));
@@ -764,8 +763,8 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
       q.resid_exact = false;
     }
   }
-  CK(launch_finalize(nullptr, nr, (const unsigned long long*)e->nmatched.p, (int64_t*)e->counts_dev.p, e->st));
-  if (counts && !counts_host) CK(cudaMemcpyAsync(counts, e->counts_dev.p, 16, cudaMemcpyDeviceToDevice, e->st));
+  CK(launch_finalize(nullptr, nr, (const unsigned long long*)e->nmatched.p, (int64_t*)e->counts_dev.p,
+                     counts && !counts_host ? counts : nullptr, e->st));
   return deliver(e, out_rc, out_mc, host_out, nr < out_cap ? nr : out_cap, counts, counts_host);
 }
 
