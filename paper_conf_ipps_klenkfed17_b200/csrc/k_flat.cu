@@ -379,18 +379,22 @@ cudaError_t launch_materialize(const Side& S, int n_ep, uint64_t* q_h, int64_t* 
 
 // ------------------------------------------------------------------ finalize
 // mm_reset: both queues' current lengths and the error flags in one launch
-__global__ void k_reset(int32_t* rlen, int32_t* mlen, int n_ep, uint32_t* err) {
+__global__ void k_reset(int32_t* rlen, int32_t* mlen, int n_ep, uint32_t* err, unsigned long long* n_matched) {
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n_ep; i += gridDim.x * blockDim.x) {
     rlen[i] = 0;
     mlen[i] = 0;
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) *err = 0u;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    *err = 0u;
+    *n_matched = 0ull;
+  }
 }
-cudaError_t launch_reset(int32_t* rlen, int32_t* mlen, int n_ep, uint32_t* err, cudaStream_t st) {
+cudaError_t launch_reset(int32_t* rlen, int32_t* mlen, int n_ep, uint32_t* err, unsigned long long* n_matched,
+                         cudaStream_t st) {
   count_launch();
   int grid = (n_ep + 255) / 256;
   if (grid > 148 * 4) grid = 148 * 4;
-  k_reset<<<grid < 1 ? 1 : grid, 256, 0, st>>>(rlen, mlen, n_ep, err);
+  k_reset<<<grid < 1 ? 1 : grid, 256, 0, st>>>(rlen, mlen, n_ep, err, n_matched);
   return cudaGetLastError();
 }
 

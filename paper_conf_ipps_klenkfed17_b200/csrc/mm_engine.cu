@@ -150,6 +150,7 @@ struct mm_engine {
   // MPI
   int64_t msg_slots = 0, warp_words = 0;
   int mpi_kernel = MM_MPI_KERNEL_FIFO;
+  bool mpi_resid_empty = true;  // no residual receive anywhere (after create / reset, before a match)
   FifoLayout fifo{};
   DBuf fifo_ws;
   // single-endpoint levels
@@ -373,7 +374,7 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
     mm_destroy(e);
     return MM_ERR_NOMEM;
   }
-  if (cudaMemsetAsync(e->err.p, 0, 4, e->st) != cudaSuccess) {
+  if (cudaMemsetAsync(e->err.p, 0, 4, e->st) != cudaSuccess || cudaMemsetAsync(e->nmatched.p, 0, 8, e->st) != cudaSuccess) {
     mm_destroy(e);
     return MM_ERR_CUDA;
   }
@@ -420,6 +421,7 @@ static int join_pending(mm_engine* e, Queue& q) {
 
 static int materialize(mm_engine* e, Queue& q, int64_t cap) {
   if (!q.pend.active) return MM_OK;
+  e->mpi_resid_empty = false;
   int jr = join_pending(e, q);
   if (jr != MM_OK) return jr;
   Side s = make_side(e, q, cap);
@@ -514,7 +516,9 @@ int mm_reset(mm_engine* e) {
   if (!e) return MM_ERR_ARG;
   LaunchScope ls(e);
   // only the current ping-pong buffer (cur = 0) is read before it is written
-  CK(launch_reset((int32_t*)e->rq.len[0].p, (int32_t*)e->mq.len[0].p, e->n_ep, (uint32_t*)e->err.p, e->st));
+  CK(launch_reset((int32_t*)e->rq.len[0].p, (int32_t*)e->mq.len[0].p, e->n_ep, (uint32_t*)e->err.p,
+                  (unsigned long long*)e->nmatched.p, e->st));
+  e->mpi_resid_empty = true;
   Queue* qs[2] = {&e->rq, &e->mq};
   for (Queue* q : qs) {
     q->pend = Pending();
@@ -568,10 +572,17 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
       if (jr != MM_OK) return jr;
     }
   Side R = make_side(e, e->rq, e->rcap), M = make_side(e, e->mq, e->mcap);
-  CK(launch_out_offsets(R, e->n_ep, (int64_t*)e->out_off.p, out_cap, (uint32_t*)e->err.p,
-                        (unsigned long long*)e->nmatched.p, e->st));  // also zeroes the pair counter
+  // With no residual receive (after a reset) the snapshot's output offsets
+  // are the posted batch's CSR offsets: no scan, and the pair counter was
+  // zeroed by mm_reset.  Otherwise one scan, which also zeroes the counter.
+  const bool direct = e->mpi_resid_empty && R.p_off && R.p_n <= out_cap;
+  const int64_t* out_off = direct ? R.p_off : (const int64_t*)e->out_off.p;
+  if (!direct)
+    CK(launch_out_offsets(R, e->n_ep, (int64_t*)e->out_off.p, out_cap, (uint32_t*)e->err.p,
+                          (unsigned long long*)e->nmatched.p, e->st));
+  e->mpi_resid_empty = false;
   if (host_out) {  // the output ranges are only known on the device: fetch them first
-    CK(cudaMemcpyAsync(e->h_off, e->out_off.p, (size_t)(e->n_ep + 1) * 8, cudaMemcpyDeviceToHost, e->st));
+    CK(cudaMemcpyAsync(e->h_off, out_off, (size_t)(e->n_ep + 1) * 8, cudaMemcpyDeviceToHost, e->st));
     CK(cudaStreamSynchronize(e->st));
   }
   MpiArgs a;
@@ -583,7 +594,7 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
   a.out_rc = drc;
   a.out_mc = dmc;
   a.out_cap = out_cap;
-  a.out_off = (const int64_t*)e->out_off.p;
+  a.out_off = out_off;
   a.q_rh_w = (uint64_t*)e->rq.hdr[0].p;
   a.q_rc_w = (int64_t*)e->rq.cookie[0].p;
   a.rres_w = (int32_t*)e->rq.len[0].p;
@@ -616,8 +627,8 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
     }
   }
   e->timer.end(e->st);
-  CK(launch_finalize((const int64_t*)e->out_off.p + e->n_ep, 0, (const unsigned long long*)e->nmatched.p,
-                     (int64_t*)e->counts_dev.p, counts && !counts_host ? counts : nullptr, e->st));
+  CK(launch_finalize(out_off + e->n_ep, 0, (const unsigned long long*)e->nmatched.p, (int64_t*)e->counts_dev.p,
+                     counts && !counts_host ? counts : nullptr, e->st));
   e->rq.pend = Pending();
   e->mq.pend = Pending();
   if (pipe) CK(cudaStreamSynchronize(e->cs));  // the caller may reuse its host inputs once we return

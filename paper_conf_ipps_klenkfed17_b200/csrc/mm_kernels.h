@@ -125,7 +125,8 @@ cudaError_t run_route(const uint64_t* a, const int64_t* b, int64_t n, int world,
                       int64_t* out_b, int64_t* counts, uint32_t* part, cudaStream_t st);
 
 // counts[] = {n_out, n_matched} from device state
-cudaError_t launch_reset(int32_t* rlen, int32_t* mlen, int n_ep, uint32_t* err, cudaStream_t st);
+cudaError_t launch_reset(int32_t* rlen, int32_t* mlen, int n_ep, uint32_t* err, unsigned long long* n_matched,
+                         cudaStream_t st);
 cudaError_t launch_finalize(const int64_t* n_out_src, int64_t n_out_host, const unsigned long long* n_matched,
                             int64_t* counts, int64_t* user_counts, cudaStream_t st);
 
