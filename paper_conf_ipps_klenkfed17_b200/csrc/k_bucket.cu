@@ -226,6 +226,25 @@ __device__ __forceinline__ uint32_t quarter_of(uint32_t x, uint32_t L) {
   return (uint32_t)(x >= L / 4) + (uint32_t)(x >= L / 2) + (uint32_t)(x >= (3 * L) / 4);
 }
 
+// Optional per-phase cycle accounting of k_bucket_pair (build with
+// -DMM_PHASE_TIMING; read by mm_debug_bucket_cycles): thread 0 adds clock64
+// deltas per phase, slot 15 counts buckets.
+#ifdef MM_PHASE_TIMING
+__device__ unsigned long long g_bucket_cycles[16];
+#define MM_BPHASE(n)                                                        \
+  do {                                                                     \
+    if (threadIdx.x == 0) {                                                \
+      const long long _t = clock64();                                      \
+      atomicAdd(&g_bucket_cycles[n], (unsigned long long)(_t - t_bphase)); \
+      t_bphase = _t;                                                       \
+    }                                                                      \
+  } while (0)
+#else
+#define MM_BPHASE(n) \
+  do {               \
+  } while (0)
+#endif
+
 __global__ void __launch_bounds__(kPairThreads, 5) k_bucket_pair(BucketArgs ba, uint32_t nbk) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   BucketSmem& sm = *reinterpret_cast<BucketSmem*>(smem_raw);
@@ -264,9 +283,13 @@ __global__ void __launch_bounds__(kPairThreads, 5) k_bucket_pair(BucketArgs ba, 
     }
   };
   uint32_t xr0, xnr, xm0, xnm;  // bounds of the bucket held in hv / iv
+#ifdef MM_PHASE_TIMING
+  long long t_bphase = clock64();
+#endif
   fetch(blockIdx.x, xr0, xnr, xm0, xnm);
   for (uint32_t b = blockIdx.x; b < nbk; b += gridDim.x) {
     __syncthreads();  // the previous bucket is done with shared memory
+    MM_BPHASE(0);
     const uint32_t r0 = xr0, nr = xnr, m0 = xm0, nm = xnm;
     const uint32_t n = nr + nm;
     if (n == 0 || n > (uint32_t)kBucketCap) {  // uniform across the CTA
@@ -287,145 +310,161 @@ __global__ void __launch_bounds__(kPairThreads, 5) k_bucket_pair(BucketArgs ba, 
     if (tid < kBucketCap / 32) sm.matched[tid] = 0u;
     if (tid == 0) sm.ntup = 0;
     fetch(b + gridDim.x, xr0, xnr, xm0, xnm);
-  __syncthreads();
-  // B: message tuples into the table; the CAS winner draws the dense id
-  for (uint32_t e = nr + tid; e < n; e += NT) {
-    const uint64_t h = sm.hdr[e];
-    const uint64_t p = h * 0xD6E8FEB86659FD93ull;
-    uint32_t s = (uint32_t)(p >> 40) & hmask;
-    const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
-    while (true) {
-      uint32_t o = sm.table[s];
-      if (o == 0xFFFFFFFFu) {
-        o = atomicCAS(&sm.table[s], 0xFFFFFFFFu, (fp << 16) | e);  // representative's header is in smem already
+    __syncthreads();
+    MM_BPHASE(1);
+    // B: message tuples into the table; the CAS winner draws the dense id
+    for (uint32_t e = nr + tid; e < n; e += NT) {
+      const uint64_t h = sm.hdr[e];
+      const uint64_t p = h * 0xD6E8FEB86659FD93ull;
+      uint32_t s = (uint32_t)(p >> 40) & hmask;
+      const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
+      while (true) {
+        uint32_t o = sm.table[s];
         if (o == 0xFFFFFFFFu) {
-          sm.sid[s] = (uint16_t)atomicAdd(&sm.ntup, 1u);
-          break;
+          o = atomicCAS(&sm.table[s], 0xFFFFFFFFu, (fp << 16) | e);  // representative's header is in smem already
+          if (o == 0xFFFFFFFFu) {
+            sm.sid[s] = (uint16_t)atomicAdd(&sm.ntup, 1u);
+            break;
+          }
         }
+        if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) break;
+        s = (s + 1) & hmask;
       }
-      if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) break;
-      s = (s + 1) & hmask;
+      sm.tup[e] = (uint16_t)s;
     }
-    sm.tup[e] = (uint16_t)s;
-  }
-  __syncthreads();
-  const uint32_t T = sm.ntup;
-  // C: tuple ids (receives look theirs up) and ranks within the side
-  if (warp < 2 * kQ) {
-    const uint32_t side = warp < kQ ? 1u : 0u, q = warp & (kQ - 1);
-    uint16_t* run = &sm.qcnt[(side * kQ + q) * kBucketCap];
-    for (uint32_t t = lane; t < T; t += 32) run[t] = 0;
-    __syncwarp();
-    const uint32_t L = side ? nm : nr, base = side ? nr : 0u;
-    const uint32_t lo = base + (q * L) / kQ, hi = base + ((q + 1) * L) / kQ;
-    const uint32_t lt = lanemask_lt();
-    for (uint32_t c = lo; c < hi; c += 32) {
-      const uint32_t e = c + lane;
+    __syncthreads();
+    MM_BPHASE(2);
+    const uint32_t T = sm.ntup;
+    // C1: tuple ids of every element (receives look theirs up); the
+    // per-quarter running counts of the T tuples cleared
+    for (uint32_t e = tid; e < n; e += NT) {
       uint32_t id = kNone;
-      if (e < hi) {
-        if (side) {
-          id = sm.sid[sm.tup[e]];
-        } else {
-          const uint64_t h = sm.hdr[e];
-          const uint64_t p = h * 0xD6E8FEB86659FD93ull;
-          uint32_t s = (uint32_t)(p >> 40) & hmask;
-          const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
-          while (true) {
-            const uint32_t o = sm.table[s];
-            if (o == 0xFFFFFFFFu) break;
-            if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) {
-              id = sm.sid[s];
-              break;
+      if (e >= nr) {
+        id = sm.sid[sm.tup[e]];
+      } else {
+        const uint64_t h = sm.hdr[e];
+        const uint64_t p = h * 0xD6E8FEB86659FD93ull;
+        uint32_t s = (uint32_t)(p >> 40) & hmask;
+        const uint32_t fp = (uint32_t)(p >> 24) & 0xFFFFu;
+        while (true) {
+          const uint32_t o = sm.table[s];
+          if (o == 0xFFFFFFFFu) break;
+          if ((o >> 16) == fp && sm.hdr[o & 0xFFFFu] == h) {
+            id = sm.sid[s];
+            break;
+          }
+          s = (s + 1) & hmask;
+        }
+      }
+      sm.tup[e] = (uint16_t)id;
+    }
+    {
+      const uint32_t T8 = (T + 7) / 8;  // 16-byte words per row
+      for (uint32_t x = tid; x < 2 * kQ * T8; x += NT)
+        reinterpret_cast<uint4*>(&sm.qcnt[(x / T8) * kBucketCap])[x % T8] = make_uint4(0u, 0u, 0u, 0u);
+    }
+    __syncthreads();
+    // C2: ranks within the side -- one warp per quarter walks it 32 elements
+    // at a time (match.any peers, per-tuple running counts)
+    if (warp < 2 * kQ) {
+      const uint32_t side = warp < kQ ? 1u : 0u, q = warp & (kQ - 1);
+      uint16_t* run = &sm.qcnt[(side * kQ + q) * kBucketCap];
+      const uint32_t L = side ? nm : nr, base = side ? nr : 0u;
+      const uint32_t lo = base + (q * L) / kQ, hi = base + ((q + 1) * L) / kQ;
+      const uint32_t lt = lanemask_lt();
+      for (uint32_t c = lo; c < hi; c += 32) {
+        const uint32_t e = c + lane;
+        const uint32_t id = e < hi ? sm.tup[e] : kNone;
+        const bool has = id != kNone;
+        const uint32_t peers = __match_any_sync(kFull, has ? id : 0x10000u + lane);
+        const uint32_t before = has ? run[id] : 0u;
+        __syncwarp();
+        if (has && (peers >> lane) == 1u) run[id] = (uint16_t)(before + __popc(peers));  // highest peer publishes
+        if (e < hi) sm.rnk[e] = (uint16_t)(before + __popc(peers & lt));
+        __syncwarp();
+      }
+    }
+    __syncthreads();
+    MM_BPHASE(3);
+    // D: per tuple -- prefixes over the quarters, message totals, and their
+    // scan (tuples TPT * tid .. TPT * tid + TPT - 1)
+    {
+      constexpr int TPT = kBucketCap / NT;  // tuples per thread
+      uint32_t tot[TPT], sum = 0;
+#pragma unroll
+      for (int j = 0; j < TPT; j++) {
+        const uint32_t t = TPT * tid + j;
+        tot[j] = 0;
+        if (t < T) {
+#pragma unroll
+          for (int side = 0; side < 2; side++) {
+            uint32_t acc = 0;
+#pragma unroll
+            for (int q = 0; q < kQ; q++) {
+              uint16_t* c = &sm.qcnt[(side * kQ + q) * kBucketCap + t];
+              const uint32_t v = *c;
+              *c = (uint16_t)acc;
+              acc += v;
             }
-            s = (s + 1) & hmask;
+            if (side) tot[j] = acc;
           }
         }
+        sum += tot[j];
       }
-      const bool has = id != kNone;
-      const uint32_t peers = __match_any_sync(kFull, has ? id : 0x10000u + lane);
-      const uint32_t before = has ? run[id] : 0u;
-      __syncwarp();
-      if (has && (peers >> lane) == 1u) run[id] = (uint16_t)(before + __popc(peers));  // highest peer publishes
-      if (e < hi) {
-        sm.tup[e] = (uint16_t)id;
-        sm.rnk[e] = (uint16_t)(before + __popc(peers & lt));
-      }
-      __syncwarp();
-    }
-  }
-  __syncthreads();
-  // D: per tuple -- prefixes over the quarters, message totals, and their
-  // scan (tuples TPT * tid .. TPT * tid + TPT - 1)
-  {
-    constexpr int TPT = kBucketCap / NT;  // tuples per thread
-    uint32_t tot[TPT], sum = 0;
+      uint32_t all;
+      uint32_t ex = block_excl_scan<uint32_t>(sum, sm.scan_sm, &all);
 #pragma unroll
-    for (int j = 0; j < TPT; j++) {
-      const uint32_t t = TPT * tid + j;
-      tot[j] = 0;
-      if (t < T) {
-#pragma unroll
-        for (int side = 0; side < 2; side++) {
-          uint32_t acc = 0;
-#pragma unroll
-          for (int q = 0; q < kQ; q++) {
-            uint16_t* c = &sm.qcnt[(side * kQ + q) * kBucketCap + t];
-            const uint32_t v = *c;
-            *c = (uint16_t)acc;
-            acc += v;
-          }
-          if (side) tot[j] = acc;
+      for (int j = 0; j < TPT; j++) {
+        const uint32_t t = TPT * tid + j;
+        if (t < T) {
+          sm.mstart[t] = (uint16_t)ex;
+          sm.mtot[t] = (uint16_t)tot[j];
         }
+        ex += tot[j];
       }
-      sum += tot[j];
     }
-    uint32_t all;
-    uint32_t ex = block_excl_scan<uint32_t>(sum, sm.scan_sm, &all);
-#pragma unroll
-    for (int j = 0; j < TPT; j++) {
-      const uint32_t t = TPT * tid + j;
-      if (t < T) {
-        sm.mstart[t] = (uint16_t)ex;
-        sm.mtot[t] = (uint16_t)tot[j];
+    __syncthreads();
+    MM_BPHASE(4);
+    // E: full ranks; messages placed by (tuple, rank)
+    for (uint32_t e = tid; e < n; e += NT) {
+      const uint32_t id = sm.tup[e];
+      if (id == kNone) continue;
+      const uint32_t side = e >= nr ? 1u : 0u;
+      const uint32_t q = side ? quarter_of(e - nr, nm) : quarter_of(e, nr);
+      const uint32_t r = sm.rnk[e] + sm.qcnt[(side * kQ + q) * kBucketCap + id];
+      if (!side) sm.rnk[e] = (uint16_t)r;
+      if (e >= nr) sm.msg_at[sm.mstart[id] + r] = (uint16_t)e;
+    }
+    __syncthreads();
+    MM_BPHASE(5);
+    // F: receives take the message of equal rank
+    uint32_t nmatch = 0;
+    for (uint32_t e = tid; e < nr; e += NT) {
+      const uint32_t id = sm.tup[e];
+      uint32_t j = kNone;
+      if (id != kNone) {
+        const uint32_t r = sm.rnk[e];
+        if (r < sm.mtot[id]) j = sm.msg_at[sm.mstart[id] + r];
       }
-      ex += tot[j];
+      int64_t mc = MM_NO_MATCH;
+      if (j != kNone) {
+        atomicOr(&sm.matched[(j - nr) >> 5], 1u << ((j - nr) & 31));
+        mc = a.M.cookie(0, sm.idx[j], mres, mpb);
+        nmatch++;
+      }
+      a.out_rc[r0 + e] = a.R.cookie(0, sm.idx[e], rres, rpb);
+      a.out_mc[r0 + e] = mc;
+      a.rflag[r0 + e] = j != kNone ? 1 : 0;
     }
-  }
-  __syncthreads();
-  // E: full ranks; messages placed by (tuple, rank)
-  for (uint32_t e = tid; e < n; e += NT) {
-    const uint32_t id = sm.tup[e];
-    if (id == kNone) continue;
-    const uint32_t side = e >= nr ? 1u : 0u;
-    const uint32_t q = side ? quarter_of(e - nr, nm) : quarter_of(e, nr);
-    const uint32_t r = sm.rnk[e] + sm.qcnt[(side * kQ + q) * kBucketCap + id];
-    if (!side) sm.rnk[e] = (uint16_t)r;
-    if (e >= nr) sm.msg_at[sm.mstart[id] + r] = (uint16_t)e;
-  }
-  __syncthreads();
-  // F: receives take the message of equal rank
-  uint32_t nmatch = 0;
-  for (uint32_t e = tid; e < nr; e += NT) {
-    const uint32_t id = sm.tup[e];
-    uint32_t j = kNone;
-    if (id != kNone) {
-      const uint32_t r = sm.rnk[e];
-      if (r < sm.mtot[id]) j = sm.msg_at[sm.mstart[id] + r];
-    }
-    int64_t mc = MM_NO_MATCH;
-    if (j != kNone) {
-      atomicOr(&sm.matched[(j - nr) >> 5], 1u << ((j - nr) & 31));
-      mc = a.M.cookie(0, sm.idx[j], mres, mpb);
-      nmatch++;
-    }
-    a.out_rc[r0 + e] = a.R.cookie(0, sm.idx[e], rres, rpb);
-    a.out_mc[r0 + e] = mc;
-    a.rflag[r0 + e] = j != kNone ? 1 : 0;
-  }
-  for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
-  if (lane == 0 && nmatch) atomicAdd(a.n_matched, (unsigned long long)nmatch);
-  __syncthreads();
-  for (uint32_t x = tid; x < nm; x += NT) a.mflag[m0 + x] = (sm.matched[x >> 5] >> (x & 31)) & 1u;
+    for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
+    if (lane == 0 && nmatch) atomicAdd(a.n_matched, (unsigned long long)nmatch);
+    MM_BPHASE(6);
+    __syncthreads();
+    for (uint32_t x = tid; x < nm; x += NT) a.mflag[m0 + x] = (sm.matched[x >> 5] >> (x & 31)) & 1u;
+#ifdef MM_PHASE_TIMING
+    MM_BPHASE(7);
+    if (threadIdx.x == 0) atomicAdd(&g_bucket_cycles[15], 1ull);
+#endif
   }
 }
 
@@ -689,3 +728,15 @@ cudaError_t run_compact_sorted(const Side& S, int64_t resid, int64_t n, const ui
 int64_t bucket_scratch_elems(int64_t n) { return ((int64_t)1 << bucket_bits_for(n)) + 1; }
 
 }  // namespace mm
+
+#ifdef MM_PHASE_TIMING
+extern "C" int mm_debug_bucket_cycles(unsigned long long* out, int reset) {
+  cudaDeviceSynchronize();
+  if (cudaMemcpyFromSymbol(out, mm::g_bucket_cycles, sizeof(unsigned long long) * 16) != cudaSuccess) return 2;
+  if (reset) {
+    unsigned long long z[16] = {0};
+    cudaMemcpyToSymbol(mm::g_bucket_cycles, z, sizeof(z));
+  }
+  return 0;
+}
+#endif
