@@ -195,7 +195,8 @@ struct BucketArgs {
 // counts), then per-tuple prefixes over the quarters complete the ranks.
 // Messages are placed by (tuple, rank) after a scan of the per-tuple message
 // counts, and the receive of rank r takes the message of rank r of its tuple.
-// O(1) work per element (no list walks, no run-length limit), 7 barriers.
+// O(1) work per element (no list walks, no run-length limit), 7 barriers;
+// message flags are written directly by the receive that takes the message.
 struct BucketSmem {
   uint64_t hdr[kBucketCap];  // receives [0, nr), then messages [nr, nr + nm)
   uint32_t idx[kBucketCap];  // snapshot index
@@ -215,7 +216,6 @@ struct BucketSmem {
   // qcnt[side][quarter][tuple]: running counts, then exclusive prefixes over
   // the quarters
   uint16_t qcnt[2 * kQ * kBucketCap];
-  uint32_t matched[kBucketCap / 32];
   uint32_t scan_sm[kPairThreads / 32 + 1];
   uint32_t ntup;
 };
@@ -307,8 +307,10 @@ __global__ void __launch_bounds__(kPairThreads, 5) k_bucket_pair(BucketArgs ba, 
       }
     }
     for (uint32_t s = tid; s < kBucketH / 4; s += NT) reinterpret_cast<uint4*>(sm.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
-    if (tid < kBucketCap / 32) sm.matched[tid] = 0u;
     if (tid == 0) sm.ntup = 0;
+    // message flags start at 0; phase F sets the matched ones (the barriers
+    // in between order the two stores)
+    for (uint32_t x = tid; x < nm; x += NT) a.mflag[m0 + x] = 0;
     fetch(b + gridDim.x, xr0, xnr, xm0, xnm);
     __syncthreads();
     MM_BPHASE(1);
@@ -448,7 +450,7 @@ __global__ void __launch_bounds__(kPairThreads, 5) k_bucket_pair(BucketArgs ba, 
       }
       int64_t mc = MM_NO_MATCH;
       if (j != kNone) {
-        atomicOr(&sm.matched[(j - nr) >> 5], 1u << ((j - nr) & 31));
+        a.mflag[m0 + (j - nr)] = 1;
         mc = a.M.cookie(0, sm.idx[j], mres, mpb);
         nmatch++;
       }
@@ -459,10 +461,7 @@ __global__ void __launch_bounds__(kPairThreads, 5) k_bucket_pair(BucketArgs ba, 
     for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
     if (lane == 0 && nmatch) atomicAdd(a.n_matched, (unsigned long long)nmatch);
     MM_BPHASE(6);
-    __syncthreads();
-    for (uint32_t x = tid; x < nm; x += NT) a.mflag[m0 + x] = (sm.matched[x >> 5] >> (x & 31)) & 1u;
 #ifdef MM_PHASE_TIMING
-    MM_BPHASE(7);
     if (threadIdx.x == 0) atomicAdd(&g_bucket_cycles[15], 1ull);
 #endif
   }
