@@ -472,7 +472,7 @@ __global__ void __launch_bounds__(kPairThreads, 5) k_bucket_pair(BucketArgs ba, 
 #endif
 // NOWILD_UNORDERED: messages pushed onto per-tuple lists, receives pop from
 // them (lock-free, pops only in that phase: no ABA) -- any maximal pairing of
-// equal tuples; 3 barriers.
+// equal tuples; 3 barriers, message flags written by the popping receive.
 struct PopSmem {
   uint64_t hdr[kBucketCap];               // receives [0, nr), then messages [nr, nr + nm)
   uint32_t idx[kBucketCap];               // snapshot index
@@ -480,7 +480,6 @@ struct PopSmem {
   uint16_t mhead[kBucketH];               // per slot: message list
   uint16_t next[kBucketCap];              // list links
   uint16_t slot[kBucketCap];              // receive -> slot | kNone
-  uint32_t matched[kBucketCap / 32];      // message matched bits (by message offset)
 };
 
 __global__ void __launch_bounds__(kBucketThreads, MM_POP_MIN_BLOCKS) k_bucket_pop(BucketArgs ba, uint32_t nbk) {
@@ -543,7 +542,9 @@ __global__ void __launch_bounds__(kBucketThreads, MM_POP_MIN_BLOCKS) k_bucket_po
       }
       for (uint32_t s = tid; s < kBucketH / 4; s += NT) reinterpret_cast<uint4*>(sm.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
       for (uint32_t s = tid; s < kBucketH / 8; s += NT) reinterpret_cast<uint4*>(sm.mhead)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
-      for (uint32_t s = tid; s < kBucketCap / 32; s += NT) sm.matched[s] = 0u;
+      // message flags start at 0; the receive that pops a message sets its
+      // flag (the barriers in between order the two stores)
+      for (uint32_t x = tid; x < nm; x += NT) a.mflag[m0 + x] = 0;
       fetch(b + gridDim.x, xr0, xnr, xm0, xnm);
     }
     __syncthreads();
@@ -602,7 +603,7 @@ __global__ void __launch_bounds__(kBucketThreads, MM_POP_MIN_BLOCKS) k_bucket_po
       }
       int64_t mc = MM_NO_MATCH;
       if (j != kNone) {
-        atomicOr(&sm.matched[(j - nr) >> 5], 1u << ((j - nr) & 31));
+        a.mflag[m0 + (j - nr)] = 1;
         mc = a.M.cookie(0, sm.idx[j], mres, mpb);
         nmatch++;
       }
@@ -612,8 +613,6 @@ __global__ void __launch_bounds__(kBucketThreads, MM_POP_MIN_BLOCKS) k_bucket_po
     }
     for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
     if (lane == 0 && nmatch) atomicAdd(a.n_matched, (unsigned long long)nmatch);
-    __syncthreads();
-    for (uint32_t x = tid; x < nm; x += NT) a.mflag[m0 + x] = (sm.matched[x >> 5] >> (x & 31)) & 1u;
   }
 }
 
