@@ -260,10 +260,13 @@ __global__ void __launch_bounds__(kPartThreads) k_part_hist(BucketF bucket, int6
 // then written out so that consecutive threads write consecutive addresses of
 // a bucket's run (coalesced stores instead of one scattered store per lane).
 // move.load(k, a, b) reads element k's payload, move.store(dst, a, b) writes it.
+#ifndef MM_PART_MIN_BLOCKS
+#define MM_PART_MIN_BLOCKS 4  // resident scatter CTAs per SM the register budget must allow (3: -6 %)
+#endif
 constexpr size_t kPartSmem = (size_t)kPartTile * (8 + 8 + 2) + (kPartWarps + 2) * kPartMaxBuckets * 4 + 64 * 4 + 16;
 
 template <class BucketF, class MoveF>
-__global__ void __launch_bounds__(kPartThreads) k_part_scatter(BucketF bucket, MoveF move, int64_t n, int nbuckets,
+__global__ void __launch_bounds__(kPartThreads, MM_PART_MIN_BLOCKS) k_part_scatter(BucketF bucket, MoveF move, int64_t n, int nbuckets,
                                                                int64_t ntiles, const uint32_t* off) {
   extern __shared__ __align__(16) uint8_t part_smem[];
   uint64_t* sa = reinterpret_cast<uint64_t*>(part_smem);
