@@ -625,16 +625,9 @@ int64_t bucket_bits_for(int64_t n) {
 }
 
 // persistent grid: every resident CTA slot of the chip, at most one per bucket
-template <class K>
-static uint32_t bucket_grid(K kernel, int threads, size_t smem, uint32_t B) {
-  int dev = 0, sms = 148, occ = 1;
-  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess ||
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, threads, smem) != cudaSuccess) {
-    cudaGetLastError();
-    sms = 148;
-    occ = 1;
-  }
-  const uint32_t g = (uint32_t)(sms * (occ < 1 ? 1 : occ));
+template <auto KERNEL>
+static uint32_t bucket_grid(int threads, size_t smem, uint32_t B) {
+  const uint32_t g = (uint32_t)resident_ctas<KERNEL>(threads, smem);
   return g < B ? g : B;
 }
 
@@ -672,16 +665,16 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cuda
   BucketArgs ba{a, rh, ri, s.roff, mh, mi, s.moff, s.overflow};
   if (ordered) {
     const size_t smem = sizeof(BucketSmem);
-    err = cudaFuncSetAttribute(k_bucket_pair, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    err = ensure_dyn_smem<k_bucket_pair>(smem);
     if (err != cudaSuccess) return err;
     count_launch();
-    k_bucket_pair<<<bucket_grid(k_bucket_pair, kPairThreads, smem, B), kPairThreads, smem, st>>>(ba, B);
+    k_bucket_pair<<<bucket_grid<k_bucket_pair>(kPairThreads, smem, B), kPairThreads, smem, st>>>(ba, B);
   } else {
     const size_t smem = sizeof(PopSmem);
-    err = cudaFuncSetAttribute(k_bucket_pop, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    err = ensure_dyn_smem<k_bucket_pop>(smem);
     if (err != cudaSuccess) return err;
     count_launch();
-    k_bucket_pop<<<bucket_grid(k_bucket_pop, kBucketThreads, smem, B), kBucketThreads, smem, st>>>(ba, B);
+    k_bucket_pop<<<bucket_grid<k_bucket_pop>(kBucketThreads, smem, B), kBucketThreads, smem, st>>>(ba, B);
   }
   return cudaGetLastError();
 }

@@ -189,7 +189,7 @@ cudaError_t launch_mpi_matrix(const MpiArgs& a, cudaStream_t st) {
   if (wpb > 8) wpb = 8;
   if (wpb < 1) wpb = 1;
   const size_t smem = per_warp * wpb;
-  cudaError_t err = cudaFuncSetAttribute(k_mpi_matrix, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t err = ensure_dyn_smem<k_mpi_matrix>(smem);
   if (err != cudaSuccess) return err;
   const int grid = (a.n_ep - a.ep0 + wpb - 1) / wpb;
   count_launch();

@@ -938,7 +938,7 @@ cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws,
   const int grid = fifo_grid(L, a.n_ep - a.ep0);
   cudaError_t err;
   if (L.in_smem) {
-    err = cudaFuncSetAttribute(k_mpi_fifo<256, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)L.total);
+    err = ensure_dyn_smem<k_mpi_fifo<256, true>>((size_t)L.total);
     if (err != cudaSuccess) return err;
     count_launch();
     k_mpi_fifo<256, true><<<grid, 256, (size_t)L.total, st>>>(a, L, nullptr);

@@ -169,6 +169,13 @@ struct mm_engine {
   cudaStream_t cs = nullptr, ds = nullptr;
   cudaEvent_t ev_st = nullptr, ev_k[kMaxChunks] = {};
   int64_t* h_off = nullptr;  // pinned copy of out_off (n_ep + 1)
+  // pinned landing zone of the small per-batch read-backs (truly asynchronous
+  // copies, no staging through pageable memory)
+  struct Small {
+    SnapInfo info;
+    unsigned long long matched;
+    uint32_t over;
+  }* h_small = nullptr;
   int pipeline = 0;          // MM_OPT_PIPELINE_CHUNKS (0 = auto)
 };
 
@@ -271,6 +278,7 @@ int mm_destroy(mm_engine* e) {
   if (e->cs) cudaStreamDestroy(e->cs);
   if (e->ds) cudaStreamDestroy(e->ds);
   if (e->h_off) cudaFreeHost(e->h_off);
+  if (e->h_small) cudaFreeHost(e->h_small);
   for (Queue* q : qs) {
     for (int b = 0; b < 2; b++) {
       release(q->hdr[b]);
@@ -316,6 +324,11 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
   }
   int rc = MM_OK;
   const bool pp = semantics != MM_SEM_MPI;
+  if (cudaMallocHost(&e->h_small, sizeof(*e->h_small)) != cudaSuccess) {
+    cudaGetLastError();
+    delete e;
+    return MM_ERR_NOMEM;
+  }
   if ((rc = alloc_queue(e, e->rq, e->rcap, pp)) != MM_OK || (rc = alloc_queue(e, e->mq, e->mcap, pp)) != MM_OK) {
     mm_destroy(e);
     return rc == MM_ERR_CUDA ? MM_ERR_NOMEM : rc;
@@ -653,8 +666,9 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
   SnapInfo info{};
   if (have_diff || !e->rq.resid_exact || !e->mq.resid_exact) {
     CK(launch_snapshot_info(R, M, bound, (SnapInfo*)e->info.p, have_diff, e->st));
-    CK(cudaMemcpyAsync(&info, e->info.p, sizeof(SnapInfo), cudaMemcpyDeviceToHost, e->st));
+    CK(cudaMemcpyAsync(&e->h_small->info, e->info.p, sizeof(SnapInfo), cudaMemcpyDeviceToHost, e->st));
     CK(cudaStreamSynchronize(e->st));
+    info = e->h_small->info;
   } else {
     info.rres = (int32_t)e->rq.resid_host;
     info.mres = (int32_t)e->mq.resid_host;
@@ -703,9 +717,11 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
     CK(run_bucketed(a, ordered, bs, e->st));
     e->timer.end(e->st);
     uint32_t over = 0;
-    CK(cudaMemcpyAsync(&over, e->bover.p, 4, cudaMemcpyDeviceToHost, e->st));
-    CK(cudaMemcpyAsync(&matched_host, e->nmatched.p, 8, cudaMemcpyDeviceToHost, e->st));
+    CK(cudaMemcpyAsync(&e->h_small->over, e->bover.p, 4, cudaMemcpyDeviceToHost, e->st));
+    CK(cudaMemcpyAsync(&e->h_small->matched, e->nmatched.p, 8, cudaMemcpyDeviceToHost, e->st));
     CK(cudaStreamSynchronize(e->st));
+    over = e->h_small->over;
+    matched_host = e->h_small->matched;
     done = over == 0;
     if (!done) {  // a bucket exceeded the on-chip capacity (heavily repeated tuples)
       e->bucket_fallbacks++;
@@ -714,8 +730,9 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
   }
   if (!done && ordered && !have_diff) {
     CK(launch_snapshot_info(R, M, bound, (SnapInfo*)e->info.p, true, e->st));
-    CK(cudaMemcpyAsync(&info, e->info.p, sizeof(SnapInfo), cudaMemcpyDeviceToHost, e->st));
+    CK(cudaMemcpyAsync(&e->h_small->info, e->info.p, sizeof(SnapInfo), cudaMemcpyDeviceToHost, e->st));
     CK(cudaStreamSynchronize(e->st));
+    info = e->h_small->info;
     have_diff = true;
   }
   if (!done && ordered) {

@@ -219,6 +219,48 @@ cudaError_t scan_apply(In in, int64_t n, T* scratch /* >= ntiles + 1 */, Out out
 
 inline int64_t scan_scratch_elems(int64_t n) { return (n + kScanTile - 1) / kScanTile + 2; }
 
+// Host-side launch helpers: the dynamic shared-memory opt-in and the
+// occupancy of a kernel are fixed per (kernel, device), so they are queried
+// once instead of on every launch (each call costs microseconds of host time
+// on the batch's critical path).
+template <auto KERNEL>
+inline cudaError_t ensure_dyn_smem(size_t bytes) {
+  static int allowed[64] = {0};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) {
+    cudaGetLastError();
+    return cudaFuncSetAttribute(KERNEL, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  }
+  if ((int)bytes <= allowed[dev]) return cudaSuccess;
+  const cudaError_t err = cudaFuncSetAttribute(KERNEL, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  if (err == cudaSuccess) allowed[dev] = (int)bytes;
+  return err;
+}
+
+// resident CTAs of KERNEL on the whole chip (SMs x blocks per SM), cached per
+// (kernel, device): every launch of a kernel uses one block size and one
+// dynamic shared-memory size
+template <auto KERNEL>
+inline int resident_ctas(int threads, size_t smem) {
+  static int cached[64] = {0};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) {
+    cudaGetLastError();
+    dev = -1;
+  }
+  if (dev >= 0 && cached[dev] > 0) return cached[dev];
+  int sms = 148, occ = 1;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev < 0 ? 0 : dev) != cudaSuccess ||
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, KERNEL, threads, smem) != cudaSuccess) {
+    cudaGetLastError();
+    sms = 148;
+    occ = 1;
+  }
+  const int r = sms * (occ < 1 ? 1 : occ);
+  if (dev >= 0) cached[dev] = r;
+  return r;
+}
+
 // ---------------------------------------------- stable bucket partition
 // Stable counting-sort scatter of n elements into up to 512 buckets.  Used by
 // the LSD radix passes of the ordered no-wildcard level (row A4) and by
@@ -395,8 +437,7 @@ cudaError_t partition_stable(BucketF bucket, MoveF move, int64_t n, int nbuckets
   uint32_t* sc = hist + m + 1;
   cudaError_t err = scan_apply<uint32_t>(ReadU32{hist}, m, sc, WriteU32{hist}, st);
   if (err != cudaSuccess) return err;
-  err = cudaFuncSetAttribute(k_part_scatter<BucketF, MoveF>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)kPartSmem);
+  err = ensure_dyn_smem<k_part_scatter<BucketF, MoveF>>(kPartSmem);
   if (err != cudaSuccess) return err;
   k_part_scatter<BucketF, MoveF><<<(unsigned)nt, kPartThreads, kPartSmem, st>>>(bucket, move, n, nbuckets, nt, hist);
   return cudaGetLastError();
