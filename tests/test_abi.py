@@ -70,3 +70,33 @@ def test_no_device_fails_loudly():
     from paper_conf_ipps_klenkfed17_b200 import Engine, MMError
     with pytest.raises(MMError):
         Engine(0, 1, 16, 16)
+
+
+def header_constants():
+    """NAME = value pairs of the enums and #defines in include/mm.h."""
+    src = re.sub(r"/\*.*?\*/", "", open(HEADER).read(), flags=re.S)
+    vals = {}
+    for body in re.findall(r"enum\s*\w*\s*\{(.*?)\}", src, flags=re.S):
+        nxt = 0
+        for item in [x.strip() for x in body.split(",") if x.strip()]:
+            m = re.match(r"(\w+)\s*(?:=\s*(-?\w+))?", item)
+            name, v = m.group(1), m.group(2)
+            nxt = int(v, 0) if v is not None else nxt
+            vals[name] = nxt
+            nxt += 1
+    for name, v in re.findall(r"#define\s+(MM_\w+)\s+\(?(-?(?:0x)?[0-9A-Fa-f]+)[uUlL]*\)?", src):
+        vals[name] = int(v, 0)
+    return vals
+
+
+def test_binding_constants_match_the_header():
+    """Every MM_* constant the Python binding defines has the header's value
+    (options, query slots, semantics levels, error codes, wildcards)."""
+    from paper_conf_ipps_klenkfed17_b200 import _lib
+    hdr = header_constants()
+    mine = {k: getattr(_lib, k) for k in dir(_lib) if k.startswith("MM_") and isinstance(getattr(_lib, k), int)}
+    common = sorted(set(hdr) & set(mine))
+    for k in ["MM_OPT_PIPELINE_CHUNKS", "MM_Q_FALLBACKS", "MM_Q_COUNT", "MM_SEM_MPI", "MM_OPT_MPI_KERNEL"]:
+        assert k in common, k
+    for k in common:
+        assert hdr[k] == mine[k], (k, hdr[k], mine[k])
