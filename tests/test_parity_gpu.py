@@ -238,6 +238,26 @@ def test_mpi_config4_worst_chain(kern):
     assert_exact(g, o)
 
 
+@pytest.mark.parametrize("case", ["worst", "mixed"])
+def test_mpi_maximum_capacity(case):
+    """Queues at the MPI level's maximum capacity (MM_MPI_MAX_MSGS, global
+    workspace variant): one endpoint 24576 deep, and 3 endpoints with mixed
+    wildcard types, two communicators and unexpected messages."""
+    from paper_conf_ipps_klenkfed17_b200._lib import MM_MPI_MAX_MSGS
+    cap = MM_MPI_MAX_MSGS
+    if case == "worst":
+        q = synth.worst_chain(seed=8, depth=cap, n_src=24, n_tag=6, lead_frac=0.1)
+        n_ep = 1
+    else:
+        q = synth.mpi_endpoints(9, n_ep=3, depth_r=cap, n_src=20, n_tag=8, p_any_src=0.02, p_any_tag=0.02,
+                                n_comm=2, ragged=False, p_unmatched=0.2)
+        n_ep = 3
+    g, qs = gpu_batches(MPI, n_ep, cap, cap, single_batch(q))
+    o, _ = oracle_batches(MPI, n_ep, single_batch(q))
+    assert_exact(g, o)
+    assert qs["error"] == 0
+
+
 @pytest.mark.slow
 @KERNELS
 def test_mpi_config1_full(kern):
