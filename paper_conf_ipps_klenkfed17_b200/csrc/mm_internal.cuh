@@ -302,12 +302,17 @@ __global__ void __launch_bounds__(kPartThreads) k_part_hist(BucketF bucket, int6
 // then written out so that consecutive threads write consecutive addresses of
 // a bucket's run (coalesced stores instead of one scattered store per lane).
 // move.load(k, a, b) reads element k's payload, move.store(dst, a, b) writes it.
+#ifndef MM_PART_ALWAYS_SENTINEL
+#define MM_PART_ALWAYS_SENTINEL 0  // 1: ten ballots per item everywhere (the previous scheme, for A/B)
+#endif
 #ifndef MM_PART_MIN_BLOCKS
 #define MM_PART_MIN_BLOCKS 4  // resident scatter CTAs per SM the register budget must allow (3: -6 %)
 #endif
 constexpr size_t kPartSmem = (size_t)kPartTile * (8 + 8 + 2) + (kPartWarps + 2) * kPartMaxBuckets * 4 + 64 * 4 + 16;
 
-template <class BucketF, class MoveF>
+// BITS: digit width (nbuckets <= 2^BITS): a full tile needs exactly BITS
+// ballots per item; the tail tile adds the sentinel bit for invalid lanes.
+template <class BucketF, class MoveF, int BITS>
 __global__ void __launch_bounds__(kPartThreads, MM_PART_MIN_BLOCKS) k_part_scatter(BucketF bucket, MoveF move, int64_t n, int nbuckets,
                                                                int64_t ntiles, const uint32_t* off) {
   extern __shared__ __align__(16) uint8_t part_smem[];
@@ -324,6 +329,7 @@ __global__ void __launch_bounds__(kPartThreads, MM_PART_MIN_BLOCKS) k_part_scatt
   __syncwarp();
   const int64_t tbase = (int64_t)blockIdx.x * kPartTile;
   const int64_t cbase = tbase + (int64_t)w * kPartWarpChunk;
+  const bool full = tbase + kPartTile <= n;  // CTA-uniform
   const uint32_t lt = lanemask_lt();
   uint32_t rank[kPartItems];
   uint32_t bk[kPartItems];
@@ -343,14 +349,21 @@ __global__ void __launch_bounds__(kPartThreads, MM_PART_MIN_BLOCKS) k_part_scatt
     bool valid = k < n;
     uint32_t b = 0;
     if (valid) b = bucket.of_payload(k, va[r], vb[r]);
-    // lanes with the same bucket: one ballot per bucket bit (here, with ten
-    // bits and eight items in flight, cheaper than match.any); invalid lanes
-    // use 512
+    // lanes with the same bucket: one ballot per digit bit (with several
+    // items in flight, cheaper than match.any); in the tail tile invalid
+    // lanes carry the sentinel value 2^BITS (one more ballot)
     uint32_t peers = kFull;
-    {
-      const uint32_t v = valid ? b : (uint32_t)kPartMaxBuckets;
+    if (full && !MM_PART_ALWAYS_SENTINEL) {
 #pragma unroll
-      for (int bit = 0; bit < 10; bit++) {
+      for (int bit = 0; bit < BITS; bit++) {
+        const bool x = (b >> bit) & 1u;
+        const uint32_t bb = __ballot_sync(kFull, x);
+        peers &= x ? bb : ~bb;
+      }
+    } else {
+      const uint32_t v = valid ? b : (1u << BITS);
+#pragma unroll
+      for (int bit = 0; bit <= BITS; bit++) {
         const bool x = (v >> bit) & 1u;
         const uint32_t bb = __ballot_sync(kFull, x);
         peers &= x ? bb : ~bb;
@@ -437,9 +450,15 @@ cudaError_t partition_stable(BucketF bucket, MoveF move, int64_t n, int nbuckets
   uint32_t* sc = hist + m + 1;
   cudaError_t err = scan_apply<uint32_t>(ReadU32{hist}, m, sc, WriteU32{hist}, st);
   if (err != cudaSuccess) return err;
-  err = ensure_dyn_smem<k_part_scatter<BucketF, MoveF>>(kPartSmem);
+  if (nbuckets <= 256 && !MM_PART_ALWAYS_SENTINEL) {
+    err = ensure_dyn_smem<k_part_scatter<BucketF, MoveF, 8>>(kPartSmem);
+    if (err != cudaSuccess) return err;
+    k_part_scatter<BucketF, MoveF, 8><<<(unsigned)nt, kPartThreads, kPartSmem, st>>>(bucket, move, n, nbuckets, nt, hist);
+    return cudaGetLastError();
+  }
+  err = ensure_dyn_smem<k_part_scatter<BucketF, MoveF, 9>>(kPartSmem);
   if (err != cudaSuccess) return err;
-  k_part_scatter<BucketF, MoveF><<<(unsigned)nt, kPartThreads, kPartSmem, st>>>(bucket, move, n, nbuckets, nt, hist);
+  k_part_scatter<BucketF, MoveF, 9><<<(unsigned)nt, kPartThreads, kPartSmem, st>>>(bucket, move, n, nbuckets, nt, hist);
   return cudaGetLastError();
 }
 
