@@ -259,6 +259,63 @@ __device__ __forceinline__ void stream_chain(const FifoWs& ws, uint32_t* kmask, 
   if (own) ws.key_c[lane] = (uint16_t)c;
 }
 
+// Wildcard chain for K <= 32 tuples (one warp, lane = tuple) over the
+// exact receives' chunk masks built by the whole CTA beforehand: kmask[c][k]
+// has bit j set if receive 32c + j is an exact receive of tuple k, kpre[c][k]
+// counts tuple k's exact receives in chunks before c.  A wildcard at posting
+// position w (chunk c, bit j) reads e_k(w) = kpre[c][k] + popc(kmask[c][k] &
+// below(j)) directly -- no walk over the receive queue --, its candidate is
+// list_k[e_k(w) + claims_k], admitted by the masked XOR (wildcard types may
+// differ here), and one redux.sync.min picks the earliest.  Software-
+// pipelined like lean_chain: the next wildcard's both candidates are loaded
+// while this step's reduction is in flight.
+template <class HdrF>
+__device__ __forceinline__ void mask_chain(const FifoWs& ws, const uint32_t* kmask, const uint16_t* kpre, uint32_t K,
+                                           uint32_t W, HdrF hdrof, int lane) {
+  const bool own = (uint32_t)lane < K;
+  uint32_t st = 0, cnt = 0;
+  uint64_t kh = 0;
+  if (own) {
+    st = ws.key_start[lane];
+    cnt = ws.key_cnt[lane];
+    kh = ws.keyhdr[lane];
+  }
+  auto exact_before = [&](uint32_t w) -> uint32_t {
+    const uint32_t ch = w >> 5, j = w & 31u;
+    return own ? (uint32_t)kpre[ch * 32 + lane] + __popc(kmask[ch * 32 + lane] & ((1u << j) - 1u)) : 0u;
+  };
+  auto head = [&](uint32_t p) { return (own && p < cnt) ? (uint32_t)ws.by_key[st + p] : 0xFFFFFFFFu; };
+  uint32_t c = 0;
+  uint32_t w = ws.wl[0];
+  uint64_t r = hdrof(0);
+  uint32_t cand = head(exact_before(w) + c);
+  for (uint32_t x = 0; x < W; x++) {
+    if (((kh ^ r) & wildcard_mask(r)) != 0) cand = 0xFFFFFFFFu;
+    const uint32_t win = __reduce_min_sync(kFull, cand);
+    // lookahead, independent of this step's outcome
+    const bool more = x + 1 < W;
+    uint32_t w2 = 0, l0 = 0xFFFFFFFFu, l1 = 0xFFFFFFFFu;
+    uint64_t r2 = 0;
+    if (more) {
+      w2 = ws.wl[x + 1];
+      r2 = hdrof(x + 1);
+      const uint32_t e2 = exact_before(w2);
+      l0 = head(e2 + c);
+      l1 = head(e2 + c + 1);
+    }
+    const bool won = win != 0xFFFFFFFFu && cand == win;
+    if (won) {
+      ws.wlog[st + c] = (uint16_t)w;
+      c++;
+    }
+    if (lane == 0) ws.recv_res[x] = win == 0xFFFFFFFFu ? kNone : (uint16_t)win;
+    cand = won ? l1 : l0;
+    w = w2;
+    r = r2;
+  }
+  if (own) ws.key_c[lane] = (uint16_t)c;
+}
+
 // The wildcard chain in its leanest form, software-pipelined.  Lane l owns
 // tuple k (own) and keeps in registers cur = its exact receives posted before
 // the current wildcard (advanced with a cursor npos over the tuple's
@@ -609,7 +666,30 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     // parallel phases of co-resident CTAs (B300_MICROARCH.md, arbiter)
     if (W > 0) {
       if (!grouped && K <= 32) {
-        if (warp == NW - 1) stream_chain(ws, ws.gnext, nr, K, W, hdrof, lane);  // gnext is free here
+        // the group arrays' space (gnext .. recv_res) is free in this path
+        const uint32_t nch = (nr + 31) / 32;
+        uint32_t* kmask = ws.gnext;
+        uint16_t* kpre = reinterpret_cast<uint16_t*>(kmask + nch * 32);
+        if ((int64_t)nch * 32 * 6 <= (int64_t)(L.recv_res - L.gnext)) {
+          for (uint32_t x = tid; x < nch * 32; x += NT) kmask[x] = 0u;
+          __syncthreads();
+          for (uint32_t i = tid; i < nr; i += NT) {
+            const uint32_t rk = ws.recv_key[i];
+            if (rk < K) atomicOr(&kmask[(i >> 5) * 32 + rk], 1u << (i & 31u));
+          }
+          __syncthreads();
+          if ((uint32_t)tid < K) {
+            uint32_t run = 0;
+            for (uint32_t ch = 0; ch < nch; ch++) {
+              kpre[ch * 32 + tid] = (uint16_t)run;
+              run += __popc(kmask[ch * 32 + tid]);
+            }
+          }
+          __syncthreads();
+          if (warp == NW - 1) mask_chain(ws, kmask, kpre, K, W, hdrof, lane);
+        } else if (warp == NW - 1) {
+          stream_chain(ws, ws.gnext, nr, K, W, hdrof, lane);  // gnext is free here
+        }
         MM_PHASE(11);
 #ifdef MM_PHASE_TIMING
         if (tid == 0) atomicAdd(&g_phase_cycles[13], 1ull);
