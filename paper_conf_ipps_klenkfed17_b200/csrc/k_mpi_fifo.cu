@@ -1022,6 +1022,12 @@ cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws,
     if (err != cudaSuccess) return err;
     count_launch();
     k_mpi_fifo<256, true><<<grid, 256, (size_t)L.total, st>>>(a, L, nullptr);
+  } else if (a.n_ep - a.ep0 <= 148) {
+    // deep queues and at most one endpoint per SM: 1024 threads per endpoint
+    // (the parallel phases over up to 24K elements shrink 4x; the chains
+    // are unchanged)
+    count_launch();
+    k_mpi_fifo<1024, false><<<grid, 1024, 0, st>>>(a, L, gws);
   } else {
     count_launch();
     k_mpi_fifo<256, false><<<grid, 256, 0, st>>>(a, L, gws);
