@@ -1013,6 +1013,9 @@ extern "C" int mm_debug_phase_cycles(unsigned long long* out, int reset) {
 }
 #endif
 
+#ifndef MM_DEEP_THREADS
+#define MM_DEEP_THREADS 1024  // threads per deep-queue endpoint CTA
+#endif
 cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws, cudaStream_t st) {
   if (a.n_ep <= a.ep0) return cudaSuccess;
   const int grid = fifo_grid(L, a.n_ep - a.ep0);
@@ -1027,7 +1030,7 @@ cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws,
     // (the parallel phases over up to 24K elements shrink 4x; the chains
     // are unchanged)
     count_launch();
-    k_mpi_fifo<1024, false><<<grid, 1024, 0, st>>>(a, L, gws);
+    k_mpi_fifo<MM_DEEP_THREADS, false><<<grid, MM_DEEP_THREADS, 0, st>>>(a, L, gws);
   } else {
     count_launch();
     k_mpi_fifo<256, false><<<grid, 256, 0, st>>>(a, L, gws);
