@@ -866,8 +866,17 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
               res = ws.recv_res[ws.recv_e[i]];
             } else if (rk != kNone) {
               const uint32_t st = ws.key_start[rk], nc = W ? ws.key_c[rk] : 0u;
-              uint32_t c = 0;
-              while (c < nc && ws.wlog[st + c] < i) c++;  // claims before i (ascending)
+              uint32_t c = 0;  // claims before i (wlog is ascending)
+              if (nc <= 8) {
+                while (c < nc && ws.wlog[st + c] < i) c++;
+              } else {  // deep queues: hundreds of claims per tuple
+                uint32_t hi = nc;
+                while (c < hi) {
+                  const uint32_t mid = (c + hi) >> 1;
+                  if (ws.wlog[st + mid] < i) c = mid + 1;
+                  else hi = mid;
+                }
+              }
               const uint32_t hd = (uint32_t)ws.recv_e[i] + c;
               if (hd < ws.key_cnt[rk]) res = ws.by_key[st + hd];
             }
