@@ -426,7 +426,13 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
   constexpr int NW = NT / 32;
   // compile-time choice, so that shared-memory accesses compile to LDS/STS/ATOMS
   uint8_t* base = SMEM ? smem_raw : gws + (size_t)blockIdx.x * L.total;
-  const FifoWs ws = carve(base, L);
+  FifoWs ws = carve(base, L);
+  if (!SMEM && L.stage_bytes > 0) {  // deep queues: the hottest arrays in shared memory
+    ws.by_key = reinterpret_cast<uint16_t*>(smem_raw + L.st_by_key);
+    ws.rby_key = reinterpret_cast<uint16_t*>(smem_raw + L.st_rby_key);
+    ws.wl = reinterpret_cast<uint16_t*>(smem_raw + L.st_wl);
+    ws.recv_key = reinterpret_cast<uint16_t*>(smem_raw + L.st_recv_key);
+  }
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t lt = lanemask_lt();
   const uint32_t H = L.H, hmask = L.H - 1;
@@ -952,6 +958,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
   }
 }
 
+constexpr int64_t kFifoStageMax = 200 * 1024;  // shared memory for the staged arrays of deep endpoints
+
 FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
   FifoLayout L;
   int64_t H = 1;
@@ -997,6 +1005,16 @@ FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
   L.recv_res = L.w_grp + r16(2 * rcap);
   L.total = off;
   L.in_smem = off <= kFifoSmemMax;
+  if (!L.in_smem) {
+    const int64_t sb = r16(2 * mcap), sr = r16(2 * rcap);
+    if (sb + 3 * sr <= kFifoStageMax) {
+      L.st_by_key = 0;
+      L.st_rby_key = sb;
+      L.st_wl = sb + sr;
+      L.st_recv_key = sb + 2 * sr;
+      L.stage_bytes = sb + 3 * sr;
+    }
+  }
   return L;
 }
 
@@ -1038,11 +1056,17 @@ cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws,
     // deep queues and at most one endpoint per SM: 1024 threads per endpoint
     // (the parallel phases over up to 24K elements shrink 4x; the chains
     // are unchanged)
+    if (L.stage_bytes > 0) {
+      err = ensure_dyn_smem<k_mpi_fifo<MM_DEEP_THREADS, false>>((size_t)L.stage_bytes);
+      if (err != cudaSuccess) return err;
+    }
     count_launch();
-    k_mpi_fifo<MM_DEEP_THREADS, false><<<grid, MM_DEEP_THREADS, 0, st>>>(a, L, gws);
+    k_mpi_fifo<MM_DEEP_THREADS, false><<<grid, MM_DEEP_THREADS, (size_t)L.stage_bytes, st>>>(a, L, gws);
   } else {
+    FifoLayout L2 = L;  // several CTAs per SM: no staging
+    L2.stage_bytes = 0;
     count_launch();
-    k_mpi_fifo<256, false><<<grid, 256, 0, st>>>(a, L, gws);
+    k_mpi_fifo<256, false><<<grid, 256, 0, st>>>(a, L2, gws);
   }
   return cudaGetLastError();
 }

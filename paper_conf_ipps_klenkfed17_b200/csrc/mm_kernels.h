@@ -34,6 +34,9 @@ struct FifoLayout {
   uint32_t H;
   uint32_t wcap;
   bool in_smem;
+  // global-workspace variant: the arrays the serial parts chase (by_key,
+  // rby_key, wl, recv_key) staged in the CTA's shared memory when they fit
+  int64_t stage_bytes = 0, st_by_key = 0, st_rby_key = 0, st_wl = 0, st_recv_key = 0;
 };
 FifoLayout fifo_layout(int64_t rcap, int64_t mcap);
 int fifo_grid(const FifoLayout& L, int n_ep);
