@@ -424,6 +424,10 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
   __shared__ uint64_t scan_sm[2][NT / 32];
   __shared__ uint32_t sh_K, sh_types, sh_matched;
   constexpr int NW = NT / 32;
+  // each side of the queue is cut in QP parts, placed by one warp each in P6
+  // (4 for 256 threads; 16 for the 1024-thread deep-endpoint CTAs)
+  constexpr int QP = NT / 64;
+  static_assert(QP >= 4 && 2 * QP <= NW, "two sides of QP parts, one warp per part");
   // compile-time choice, so that shared-memory accesses compile to LDS/STS/ATOMS
   uint8_t* base = SMEM ? smem_raw : gws + (size_t)blockIdx.x * L.total;
   FifoWs ws = carve(base, L);
@@ -451,9 +455,18 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     }
     const uint32_t nr = (uint32_t)nr64, nm = (uint32_t)nm64;
     const EpSide RS(a.R, e, rres, rpb), MS(a.M, e, mres, mpb);
-    // quarter boundaries: element x is in quarter q iff qb[q] <= x < qb[q + 1]
+    // part boundaries: element x of a side of n is in part q = x * QP / n,
+    // i.e. ceil(n q / QP) <= x < ceil(n (q + 1) / QP) (QP = 4: three compares)
     const uint32_t mq1 = (nm + 3) / 4, mq2 = (2 * nm + 3) / 4, mq3 = (3 * nm + 3) / 4;
     const uint32_t rq1 = (nr + 3) / 4, rq2 = (2 * nr + 3) / 4, rq3 = (3 * nr + 3) / 4;
+    auto mpart = [&](uint32_t j) -> uint32_t {
+      if (QP == 4) return (j >= mq1) + (j >= mq2) + (j >= mq3);
+      return (uint32_t)(((uint64_t)j * QP) / nm);
+    };
+    auto rpart = [&](uint32_t i) -> uint32_t {
+      if (QP == 4) return (i >= rq1) + (i >= rq2) + (i >= rq3);
+      return (uint32_t)(((uint64_t)i * QP) / nr);
+    };
     MM_PHASE(0);
     // the first round of message headers is requested before P1, so their
     // HBM latency overlaps the table clearing and the barrier
@@ -468,7 +481,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     for (uint32_t s = tid; s < H / 4; s += NT) reinterpret_cast<uint4*>(ws.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
     for (uint32_t k = tid; k < (nm + 31) / 32; k += NT) ws.matched[k] = 0u;
     if (SMEM) {  // per-quarter counts cleared in bulk (in HBM the CAS winners clear their rows)
-      const uint32_t n16 = (uint32_t)(8 * ws.mcap * 2 / 16);
+      const uint32_t n16 = (uint32_t)(2 * QP * ws.mcap * 2 / 16);
       for (uint32_t s = tid; s < n16; s += NT) reinterpret_cast<uint4*>(ws.pcnt)[s] = make_uint4(0u, 0u, 0u, 0u);
     }
     if (tid == 0) {
@@ -506,7 +519,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
               ws.keyhdr[id] = h;
               if (!SMEM) {
 #pragma unroll
-                for (int q = 0; q < 8; q++) ws.pcnt[q * ws.mcap + id] = 0;
+                for (int q = 0; q < 2 * QP; q++) ws.pcnt[q * ws.mcap + id] = 0;
               }
               ws.key_c[id] = 0;
               __threadfence_block();
@@ -524,8 +537,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           s = (s + 1) & hmask;
         }
         ws.msg_key[j] = (uint16_t)id;
-        const uint32_t q = (j >= mq1) + (j >= mq2) + (j >= mq3);
-        inc16(&ws.pcnt[q * ws.mcap + id]);
+        inc16(&ws.pcnt[mpart(j) * ws.mcap + id]);
       }
     }
     // the first round of receive headers, requested before the barrier
@@ -570,8 +582,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             s = (s + 1) & hmask;
           }
           if (rk != kNone) {
-            const uint32_t q = 4 + (i >= rq1) + (i >= rq2) + (i >= rq3);
-            inc16(&ws.pcnt[q * ws.mcap + rk]);
+            inc16(&ws.pcnt[(QP + rpart(i)) * ws.mcap + rk]);
           }
         }
         ws.recv_key[i] = rk;
@@ -590,13 +601,13 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       const uint32_t k0 = min(K, tid * per), k1 = min(K, k0 + per);
       uint32_t c = 0;
       for (uint32_t k = k0; k < k1; k++) {
-        // exclusive prefix over the quarters: the base rank of each quarter
+        // exclusive prefix over the parts: the base rank of each part
         uint32_t rm = 0, rr = 0;
 #pragma unroll
-        for (int q = 0; q < 4; q++) {
-          const uint32_t x = ws.pcnt[q * ws.mcap + k], y = ws.pcnt[(4 + q) * ws.mcap + k];
+        for (int q = 0; q < QP; q++) {
+          const uint32_t x = ws.pcnt[q * ws.mcap + k], y = ws.pcnt[(QP + q) * ws.mcap + k];
           ws.pcnt[q * ws.mcap + k] = (uint16_t)rm;
-          ws.pcnt[(4 + q) * ws.mcap + k] = (uint16_t)rr;
+          ws.pcnt[(QP + q) * ws.mcap + k] = (uint16_t)rr;
           rm += x;
           rr += y;
         }
@@ -637,13 +648,13 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     };
     MM_PHASE(5);
     // P6 -------------------------------------------------------------------
-    // warps 0-3 place the four quarters of the messages, warps 4-7 the four
-    // quarters of the receives; each quarter starts from its base ranks
-    if (warp < 8) {
-      const bool msg_side = warp < 4;
-      const int q = warp & 3;
+    // warps 0..QP-1 place the QP parts of the messages, warps QP..2QP-1
+    // those of the receives; each part starts from its base ranks
+    if (warp < 2 * QP) {
+      const bool msg_side = warp < QP;
+      const int q = warp % QP;
       const uint32_t n = msg_side ? nm : nr;
-      const uint32_t x0 = (n * q + 3) / 4, x1 = (n * (q + 1) + 3) / 4;
+      const uint32_t x0 = (uint32_t)(((uint64_t)n * q + QP - 1) / QP), x1 = (uint32_t)(((uint64_t)n * (q + 1) + QP - 1) / QP);
       uint16_t* running = ws.pcnt + (int64_t)warp * ws.mcap;
       if (msg_side) {
         place_in_order(
@@ -996,7 +1007,11 @@ FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
   // and group arrays (P7..P8)
   const int64_t gn = r16(4 * mcap) > 128 ? r16(4 * mcap) : 128;  // gnext; also the K <= 32 chain's kmask[32]
   const int64_t grp = gn + 2 * r16(4 * mcap) + 2 * r16(2 * rcap);
-  const int64_t region = take(grp > 16 * mcap ? grp : 16 * mcap);
+  // per-part counts: 2 sides x 4 parts (on chip) or x 16 parts (global
+  // workspace, 1024-thread deep-endpoint CTAs)
+  const int64_t rows8 = grp > 16 * mcap ? grp : 16 * mcap;
+  const bool fits = off + rows8 <= kFifoSmemMax;
+  const int64_t region = take(fits ? rows8 : (grp > 64 * mcap ? grp : 64 * mcap));
   L.pcnt = region;
   L.gnext = region;
   L.gfirst = region + gn;
