@@ -328,9 +328,10 @@ __device__ __forceinline__ void mask_chain(const FifoWs& ws, const uint32_t* kma
 // a win at step t --, so a step's critical path is the reduction and a select.
 // ADMIT: wildcards may differ in type, so each lane tests admission with the
 // masked XOR.
-template <bool ADMIT, class InF, class HdrF>
+template <bool ADMIT, class HdrF>
 __device__ __forceinline__ void lean_chain(const FifoWs& ws, bool own, uint32_t k, uint32_t x_begin, uint32_t W,
-                                           uint32_t left, InF in_chain, HdrF hdrof, int lane) {
+                                           uint32_t left, const uint16_t* grp_of, uint32_t gg, HdrF hdrof,
+                                           int lane) {
   if (left == 0) return;
   uint32_t st = 0, hend = 0, rs = 0, rc = 0;
   uint64_t kh = 0;
@@ -356,15 +357,29 @@ __device__ __forceinline__ void lean_chain(const FifoWs& ws, bool own, uint32_t 
       np3 = rpos(cur + 3);
     }
   };
-  // cursor over the chain's wildcards (warp-uniform)
+  // cursor over the chain's wildcards (warp-uniform), 32 positions a chunk:
+  // the next chunk's group ids, positions (and headers) are loaded while the
+  // current one is served
   uint32_t cb = x_begin & ~31u, cm = 0, wv = 0;
   uint64_t rv = 0;
-  auto load_chunk = [&]() {
-    const uint32_t y = cb + lane;
-    const bool in = y >= x_begin && y < W && in_chain(y);
+  uint32_t pg = kNone, pw = 0;
+  uint64_t pr = 0;
+  auto prefetch = [&](uint32_t base) {
+    const uint32_t y = base + lane;
+    const bool ok = y >= x_begin && y < W;
+    pg = ok ? (uint32_t)grp_of[y] : kNone;
+    pw = ok ? (uint32_t)ws.wl[y] : 0u;
+    if (ADMIT) pr = ok ? hdrof(y) : 0ull;
+  };
+  auto commit = [&]() {  // the prefetched chunk becomes current
+    const bool in = pg == gg;
     cm = __ballot_sync(kFull, in);
-    wv = in ? (uint32_t)ws.wl[y] : 0u;
-    if (ADMIT) rv = in ? hdrof(y) : 0ull;
+    wv = in ? pw : 0u;
+    if (ADMIT) rv = in ? pr : 0ull;
+  };
+  auto load_chunk = [&]() {
+    commit();
+    prefetch(cb + 32);
   };
   auto next = [&](uint32_t& w, uint32_t& y, uint64_t& r) {
     while (cm == 0) {
@@ -377,6 +392,7 @@ __device__ __forceinline__ void lean_chain(const FifoWs& ws, bool own, uint32_t 
     y = cb + bit;
     if (ADMIT) r = __shfl_sync(kFull, rv, bit);
   };
+  prefetch(cb);
   load_chunk();
   uint32_t w, y;
   uint64_t r = 0;
@@ -829,9 +845,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             // the group's wildcards in posting order, from its first one
             const uint32_t left = ws.gwc[gg];
             const uint32_t x0 = b + l;
-            auto in_group = [&](uint32_t y) { return ws.w_grp[y] == gg; };
             if (kn <= 32) {
-              lean_chain<false>(ws, lane < (int)kn, mine, x0, W, left, in_group, hdrof, lane);
+              lean_chain<false>(ws, lane < (int)kn, mine, x0, W, left, ws.w_grp, gg, hdrof, lane);
             } else {  // a group of more than 32 tuples: scan every tuple, admission tested
               for (uint32_t xx = x0; xx < W; xx++)
                 if (ws.w_grp[xx] == gg) {
