@@ -21,4 +21,6 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_p
     python bench.py --steps 1 --warmup 3 --levels ordered,unordered --no-cpu-baseline > gpurun_out/ncu_flat_$TAG.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_bucket_pop" -s 2 -c 1 -o gpurun_out/prof_pop_$TAG \
     python bench.py --steps 1 --warmup 3 --levels unordered --no-cpu-baseline > gpurun_out/ncu_pop_$TAG.log 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:"k_mpi_fifo" -s 2 -c 1 -o gpurun_out/prof_deep_$TAG \
+    python bench.py --steps 1 --warmup 3 --levels mpi_worst --no-cpu-baseline > gpurun_out/ncu_deep_$TAG.log 2>&1
 ls gpurun_out | grep $TAG

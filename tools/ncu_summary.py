@@ -2,7 +2,9 @@
 """Summarise ncu outputs into profiles/ (run here, on the CPU box).
 
     python tools/ncu_summary.py launches <launches.csv> <out.md>
-    python tools/ncu_summary.py full <prof.ncu-rep> <out.md> [--traffic profiles/kernel_traffic.json]
+    python tools/ncu_summary.py full <prof.ncu-rep> <out.md> [--traffic profiles/kernel_traffic.json] [--key NAME]
+    (--key stores the capture's counters under NAME instead of the kernel's
+    short name, e.g. k_mpi_fifo_deep for the configs[4] launch)
 
 `launches`: per-kernel launch counts, summed/avg device time and share of the
 step (ncu --metrics gpu__time_duration.sum, cold-cache & serialised: shares,
@@ -63,7 +65,7 @@ def launches(path, out):
     print("\n".join(lines[:25]))
 
 
-def full(path, out, traffic=None):
+def full(path, out, traffic=None, key=None):
     raw = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(raw)))
     h, units = rows[0], rows[1]
@@ -110,7 +112,7 @@ def full(path, out, traffic=None):
         old = json.load(open(traffic)) if __import__("os").path.exists(traffic) else {}
         for k, d in tr.items():
             n = d["launches"]
-            old[k] = {"dram_bytes_per_launch": d["dram_bytes"] / n, "warp_inst_per_launch": d["inst"] / n,
+            old[key or k] = {"dram_bytes_per_launch": d["dram_bytes"] / n, "warp_inst_per_launch": d["inst"] / n,
                       "issue_active_pct": d["issue"] / n, "source": path.split("/")[-1]}
         json.dump(old, open(traffic, "w"), indent=1)
 
@@ -121,4 +123,5 @@ if __name__ == "__main__":
         launches(sys.argv[2], sys.argv[3])
     else:
         tr = sys.argv[sys.argv.index("--traffic") + 1] if "--traffic" in sys.argv else None
-        full(sys.argv[2], sys.argv[3], tr)
+        key = sys.argv[sys.argv.index("--key") + 1] if "--key" in sys.argv else None
+        full(sys.argv[2], sys.argv[3], tr, key)
