@@ -79,17 +79,21 @@ def load_traffic(kernel, key="dram_bytes_per_launch"):
     return v.get(key) if isinstance(v, dict) else None
 
 
-def issue_efficiency(kernel, kernel_ms, sm_mhz):
+def issue_efficiency(kernel, kernel_ms, sm_mhz, sms_used=None):
     """Warp-issue efficiency of `kernel` (north_star: "warp-issue efficiency"):
     its warp instructions per launch (ncu capture) over the live kernel time,
     against the issue peak of 4 warp instructions per SM per clock (one per
     SM sub-partition) x SMs x the sampled SM clock; plus ncu's own
-    issue-active percentage of the captured launch."""
+    issue-active percentage of the captured launch.  `sms_used` (a launch
+    that occupies fewer SMs than the chip, e.g. configs[4]'s single endpoint
+    CTA) scales the peak to the SMs the launch can use."""
     import torch
     inst = load_traffic(kernel, "warp_inst_per_launch")
     if not inst or not kernel_ms:
         return None
     sms = torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
+    if sms_used:
+        sms = min(sms, sms_used)
     peak = 4.0 * sms * sm_mhz * 1e6 / 1e9
     ach = inst / (kernel_ms / 1e3) / 1e9
     return {"kernel": kernel, "warp_inst_per_launch": inst, "achieved": ach, "peak": peak,
@@ -265,7 +269,7 @@ def bench_mpi_worst(args, world, rank, peak):
     # ncu counters of the 1024-thread deep-endpoint launch are keyed apart from
     # the configs[1] launch (same kernel name, different instantiation and work)
     res.update(matches_per_step=matches, algo_bytes=8 * 2 * n + 16 * n, n_recv=n, n_msg=n, kernel="k_mpi_fifo",
-               capture="k_mpi_fifo_deep")
+               capture="k_mpi_fifo_deep", sms_used=1)
     eng.close()
     out = finish_level(res, world, peak, "mpi_worst")
     out["_kernel_only"] = True
@@ -365,6 +369,7 @@ def finish_level(res, world, peak, level):
                      "traffic": load_traffic(res.get("capture", res["kernel"])),
                      "kernel_ms": kernel_ms, "algo_bytes_per_launch": res["algo_bytes"]},
         "_t_ms": res["t_ms"], "_launches": res.get("launches"), "_capture": res.get("capture", res["kernel"]),
+        "_sms_used": res.get("sms_used"),
     }
     if "e2e" in res:
         out["e2e"] = res["e2e"]
@@ -477,7 +482,7 @@ def main():
         rf = lv["roofline"]
         if rf.get("kernel", "").startswith("k_mpi"):
             lv["issue"] = issue_efficiency(lv.get("_capture", rf["kernel"]), rf.get("kernel_ms"),
-                                           ck.get("sm_max_mhz") or 1965.0)
+                                           ck.get("sm_max_mhz") or 1965.0, lv.get("_sms_used"))
     head = levels.get("mpi") or next(iter(levels.values()))
     line = {
         "metric": METRIC, "value": head["value"], "unit": "matches/s", "n_gpus": world, "steps": args.steps,
