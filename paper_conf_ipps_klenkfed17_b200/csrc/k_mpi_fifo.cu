@@ -342,7 +342,8 @@ __device__ __forceinline__ void lean_chain(const FifoWs& ws, bool own, uint32_t 
     rc = ws.key_rcnt[k];
     if (ADMIT) kh = ws.keyhdr[k];
   }
-  uint32_t cur = 0, c = 0;
+  // claims already made on k (a group's leading run, lead_run) -- 0 otherwise
+  uint32_t cur = 0, c = own ? (uint32_t)ws.key_c[k] : 0u;
   // the next four exact-receive positions of k in registers: the cursor
   // advances without waiting on a shared-memory load per step
   auto rpos = [&](uint32_t x) { return x < rc ? (uint32_t)ws.rby_key[rs + x] : 0xFFFFFFFFu; };
@@ -426,6 +427,110 @@ __device__ __forceinline__ void lean_chain(const FifoWs& ws, bool own, uint32_t 
   }
   if (own) ws.key_c[k] = (uint16_t)c;
 }
+
+// position of the n-th (0-based) set bit of b (n < popc(b))
+__device__ __forceinline__ uint32_t nth_set(uint32_t b, uint32_t n) {
+  uint32_t p = 0;
+#pragma unroll
+  for (uint32_t s = 16; s; s >>= 1)
+    if ((uint32_t)__popc(b & ((1u << (p + s)) - 1u)) <= n) p += s;
+  return p;
+}
+
+// Leading run of a wildcard group.  The group's wildcards
+// posted before the first exact receive of any of its tuples (position fe)
+// see every tuple of the group with no exact receive ahead of them
+// (e_k(w) = 0), and the group's tuples are exactly the ones they admit; so
+// the r-th of them takes the group's r-th message in arrival order -- the
+// earliest unmatched admissible message (§II.B l.65-67) -- and the
+// run is a merge of two ordered streams (the run's wildcards in posting
+// order, the group's messages in queue order), 32 pairs a step, instead of a
+// chain of min-reductions.  The claims are logged per tuple exactly as the
+// chain logs them (wlog, key_c), so lean_chain continues with the group's
+// later wildcards.  Needs msg_key alive in P7 (its own wlog region: global
+// workspace).  Returns the number of pairs; x_next = the first wildcard
+// position the chain has to continue from.
+template <class MsgHdrF>
+__device__ __forceinline__ uint32_t lead_run(const FifoWs& ws, uint32_t fe, uint32_t x_begin, uint32_t W,
+                                             uint32_t nm, uint32_t gg, uint64_t gmsk, MsgHdrF mhdr, int lane,
+                                             uint32_t& x_next) {
+  const uint32_t lt = lanemask_lt();
+  const uint64_t gh = ws.keyhdr[gg] & gmsk;
+  uint32_t xc = x_begin, jc = 0, wx = 0, nw = 0, mj = 0, nq = 0, paired = 0;
+  bool wdone = false, mdone = nm == 0;
+  // append to a lane-aligned window the positions whose bit is set in the
+  // 32-wide chunks at cur, cur + 32, ... (four chunks loaded at once); a stop
+  // bit ends the stream at its position
+  auto fill = [&](uint32_t& win, uint32_t& n, uint32_t& cur, bool& done, uint32_t lim, auto pred) {
+    while (!done && n < 32) {
+      uint32_t bs[4], ss[4];
+#pragma unroll
+      for (int u = 0; u < 4; u++) {
+        bool in, stop;
+        pred(cur + 32 * u + lane, in, stop);
+        bs[u] = __ballot_sync(kFull, in);
+        ss[u] = __ballot_sync(kFull, stop);
+      }
+#pragma unroll
+      for (int u = 0; u < 4; u++) {
+        if (done || n >= 32) break;
+        const uint32_t base = cur;
+        uint32_t b = bs[u];
+        const uint32_t stop = ss[u];
+        if (stop) b &= (stop & (0u - stop)) - 1u;  // the bits below the first stop
+        const uint32_t nb = __popc(b), take = min(nb, 32u - n);
+        if ((uint32_t)lane >= n && (uint32_t)lane < n + take) win = base + nth_set(b, (uint32_t)lane - n);
+        n += take;
+        if (take < nb) {
+          cur = base + nth_set(b, take - 1) + 1;  // window full
+        } else if (stop) {
+          cur = base + (uint32_t)(__ffs(stop) - 1);
+          done = true;
+        } else {
+          cur = base + 32;
+          if (cur >= lim) done = true;
+        }
+      }
+    }
+  };
+  while (true) {
+    fill(wx, nw, xc, wdone, W, [&](uint32_t x, bool& in, bool& stop) {
+      const bool g = x < W && ws.w_grp[x] == gg;
+      const bool run = g && ws.wl[x] < fe;
+      in = run;
+      stop = g && !run;
+    });
+    fill(mj, nq, jc, mdone, nm, [&](uint32_t j, bool& in, bool& stop) {
+      in = j < nm && (mhdr(j) & gmsk) == gh;
+      stop = false;
+    });
+    const uint32_t n = min(nw, nq);
+    if (n == 0) break;  // the run ended, or the group's messages did
+    const bool act = (uint32_t)lane < n;
+    const uint32_t k = act ? (uint32_t)ws.msg_key[mj] : 0xFFFFFFFFu;
+    const uint32_t peers = __match_any_sync(kFull, k);
+    const uint32_t c0 = act ? (uint32_t)ws.key_c[k] : 0u;
+    __syncwarp();
+    if (act) {
+      const uint32_t c = c0 + __popc(peers & lt);  // claims on k in pairing order
+      ws.recv_res[wx] = (uint16_t)mj;
+      ws.wlog[ws.key_start[k] + c] = ws.wl[wx];
+      if ((peers >> lane) == 1u) ws.key_c[k] = (uint16_t)(c + 1);
+    }
+    __syncwarp();
+    paired += n;
+    wx = __shfl_down_sync(kFull, wx, n & 31u);
+    mj = __shfl_down_sync(kFull, mj, n & 31u);
+    nw -= n;
+    nq -= n;
+  }
+  x_next = nw ? __shfl_sync(kFull, wx, 0) : xc;
+  return paired;
+}
+
+#ifndef MM_LEAD_MIN
+#define MM_LEAD_MIN 8  // a group's wildcards from which a leading run is looked for
+#endif
 
 // wildcards of one type use the group chains above this many tuples (below,
 // one warp walks the receive queue: stream_chain)
@@ -735,6 +840,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         // touch disjoint tuple groups {k : k & mask == r & mask}; groups are
         // independent and run on different warps, each group's wildcards in
         // posting order.
+        // leading runs need msg_key in P7: only with wlog in a region of its own
+        const bool lead_ok = !SMEM && ws.wlog != ws.msg_key;
         const uint32_t code = __ffs(types) - 1;
         const uint64_t gmsk = (code & 1 ? ~0xFFFFFFFFull : ~0ull) & (code & 2 ? ~(0xFFFFull << 32) : ~0ull);
         // group table: the first tuple of a group to win a slot represents it;
@@ -843,9 +950,20 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
               node = ws.gnext[node];
             }
             // the group's wildcards in posting order, from its first one
-            const uint32_t left = ws.gwc[gg];
-            const uint32_t x0 = b + l;
+            uint32_t left = ws.gwc[gg];
+            uint32_t x0 = b + l;
             if (kn <= 32) {
+              if (lead_ok && left >= MM_LEAD_MIN) {
+                // first exact receive of any of the group's tuples
+                uint32_t fe = 0xFFFFFFFFu;
+                if (lane < (int)kn && ws.key_rcnt[mine]) fe = ws.rby_key[ws.key_rstart[mine]];
+                fe = __reduce_min_sync(kFull, fe);
+                uint32_t xn;
+                const uint32_t np = lead_run(ws, fe, x0, W, nm, gg, gmsk, [&](uint32_t j) { return MS.hdr(j); },
+                                             lane, xn);
+                left -= np;
+                x0 = xn;
+              }
               lean_chain<false>(ws, lane < (int)kn, mine, x0, W, left, ws.w_grp, gg, hdrof, lane);
             } else {  // a group of more than 32 tuples: scan every tuple, admission tested
               for (uint32_t xx = x0; xx < W; xx++)
@@ -1033,8 +1151,11 @@ FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
   L.gwc = L.gfirst + r16(4 * mcap);
   L.w_grp = L.gwc + r16(4 * mcap);
   L.recv_res = L.w_grp + r16(2 * rcap);
-  L.total = off;
   L.in_smem = off <= kFifoSmemMax;
+  // global workspace: wlog in a region of its own, so that msg_key stays
+  // alive in P7 for the groups' leading runs (lead_run)
+  if (!L.in_smem) L.wlog = take(2 * mcap);
+  L.total = off;
   if (!L.in_smem) {
     const int64_t sb = r16(2 * mcap), sr = r16(2 * rcap);
     if (sb + 3 * sr <= kFifoStageMax) {

@@ -212,6 +212,40 @@ def worst_chain(seed=4, depth=16384, n_src=16, n_tag=4, lead_frac=0.25):
     return Queues(pack(rsrc, rtag), off, pack(msrc, mtag), off, "worst_chain")
 
 
+def lead_runs(seed, n_ep=1, depth=4096, n_src=12, n_tag=5, lead=1024, kind="src", p_wild_after=0.05,
+              msg_frac=1.0, ragged=False):
+    """Endpoints whose receive queues START with a run of wildcard receives of
+    one type (kind "src": (ANY_SOURCE, tag); "tag": (src, ANY_TAG)) followed
+    by exact receives with a p_wild_after share of wildcards of the same type;
+    msg_frac < 1 gives fewer messages than receives (some wildcard groups run
+    out of messages inside the leading run).  Exercises the global-workspace
+    kernel's leading-run path next to the chains."""
+    rng = np.random.default_rng(seed)
+    rs, ms, ro, mo = [], [], [0], [0]
+    for _ in range(n_ep):
+        nr = int(rng.integers(depth // 2, depth + 1)) if ragged else depth
+        nm = int(msg_frac * nr)
+        src = rng.integers(0, n_src, nr)
+        tag = rng.integers(0, n_tag, nr)
+        mi = rng.permutation(nr)[:nm]
+        msrc, mtag = src[mi], tag[mi]
+        rsrc, rtag = src.copy(), tag.copy()
+        nl = min(lead, nr)
+        after = np.zeros(nr, dtype=bool)
+        after[nl:] = rng.random(nr - nl) < p_wild_after
+        wild = after.copy()
+        wild[:nl] = True
+        if kind == "src":
+            rsrc[wild] = ANY_SOURCE
+        else:
+            rtag[wild] = ANY_TAG
+        rs.append(pack(rsrc, rtag))
+        ms.append(pack(msrc, mtag))
+        ro.append(ro[-1] + nr)
+        mo.append(mo[-1] + nm)
+    return Queues(np.concatenate(rs), ro, np.concatenate(ms), mo, "lead_runs")
+
+
 def random_case(seed, n_ep=3, max_depth=40, wild=True, n_src=4, n_tag=4, n_comm=2):
     """Small irregular case for property tests (ragged depths, empty queues,
     several communicators, optional wildcards, unexpected messages)."""

@@ -258,6 +258,42 @@ def test_mpi_maximum_capacity(case):
     assert qs["error"] == 0
 
 
+@pytest.mark.parametrize("case", [
+    dict(seed=1, depth=4096, lead=1024, kind="src"),
+    dict(seed=2, depth=4096, lead=1000, kind="tag", n_src=40, n_tag=3),
+    dict(seed=3, depth=3000, lead=2500, kind="src", msg_frac=0.5),   # groups run dry inside the run
+    dict(seed=4, depth=2048, lead=37, kind="src", p_wild_after=0.3),
+    dict(seed=5, depth=2048, lead=700, kind="tag", n_src=3, n_tag=50, p_wild_after=0.2),
+    dict(seed=6, depth=5000, lead=5000, kind="src", n_tag=2),         # receives are all wildcards
+], ids=lambda c: "s%d" % c["seed"])
+def test_mpi_leading_wildcard_runs(case):
+    """Wildcard runs ahead of every exact receive of their group, on the
+    1024-thread deep-endpoint kernel (leading-run merge, then the chains)."""
+    c = dict(case)
+    q = synth.lead_runs(c.pop("seed"), **c)
+    cap = int(max(np.diff(q.recv_off).max(), np.diff(q.msg_off).max(), 1))
+    g, qs = gpu_batches(MPI, q.n_endpoints, cap, cap, single_batch(q))
+    o, _ = oracle_batches(MPI, q.n_endpoints, single_batch(q))
+    assert_exact(g, o)
+    assert qs["error"] == 0
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_mpi_leading_runs_many_endpoints_multibatch(seed):
+    """Leading runs on the 256-thread global-workspace kernel (more endpoints
+    than SMs, queues too deep for shared memory), over 3 batches with
+    residual queues (a residual UMQ ahead of the new messages)."""
+    rng = np.random.default_rng(seed)
+    q = synth.lead_runs(seed + 20, n_ep=160, depth=2048, lead=300, kind="src" if seed % 2 else "tag",
+                        msg_frac=0.8, ragged=True, n_src=10, n_tag=6)
+    batches = split_batches(q, 3, rng)
+    g, qs = gpu_batches(MPI, q.n_endpoints, 2048, 2048, batches)
+    o, oe = oracle_batches(MPI, q.n_endpoints, batches)
+    assert_exact(g, o)
+    rr, rm = oe.residual_depths()
+    assert qs["resid_recv"] == sum(rr) and qs["resid_msg"] == sum(rm)
+
+
 @pytest.mark.slow
 @KERNELS
 def test_mpi_config1_full(kern):
