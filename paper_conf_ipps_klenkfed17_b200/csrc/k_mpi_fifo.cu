@@ -848,6 +848,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         // it initialises its group entries BEFORE publishing, so members that
         // find it may link themselves in at once (no pending state)
         for (uint32_t k = tid; k < K; k += NT) {
+          ws.gwc[k] = 0;  // every tuple: nonzero after the wildcard pass = a representative with wildcards
           const uint64_t gk = ws.keyhdr[k] & gmsk;
           uint32_t s, fp;
           slot_fp(gk, hmask, s, fp);
@@ -928,12 +929,12 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         }
         __syncthreads();
         MM_PHASE(10);
-        // warp v serves the groups whose first wildcard it finds with g % NW == v
+        // warp v serves the groups g % NW == v that still have wildcards (the
+        // representatives are enumerated directly: no scan of the wildcards)
         const uint32_t v = (uint32_t)(NW - 1 - warp);
-        for (uint32_t b = 0; b < W; b += 32) {
-          const uint32_t x = b + lane;
-          const uint32_t g = x < W ? ws.w_grp[x] : kNone;
-          const bool lead = g != kNone && g % NW == v && ws.gfirst[g] == x && ws.gwc[g] != 0;
+        for (uint32_t b = v; b < K; b += 32 * NW) {
+          const uint32_t g = b + (uint32_t)lane * NW;
+          const bool lead = g < K && ws.gwc[g] != 0;
           uint32_t leaders = __ballot_sync(kFull, lead);
           while (leaders) {
             const int l = __ffs(leaders) - 1;
@@ -951,7 +952,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             }
             // the group's wildcards in posting order, from its first one
             uint32_t left = ws.gwc[gg];
-            uint32_t x0 = b + l;
+            uint32_t x0 = ws.gfirst[gg];
             if (kn <= 32) {
               if (lead_ok && left >= MM_LEAD_MIN) {
                 // first exact receive of any of the group's tuples
