@@ -428,6 +428,10 @@ __device__ __forceinline__ void lean_chain(const FifoWs& ws, bool own, uint32_t 
   if (own) ws.key_c[k] = (uint16_t)c;
 }
 
+#ifndef MM_LEAD_CHUNKS
+#define MM_LEAD_CHUNKS 2  // 32-wide chunks a leading run loads per stream at once
+#endif
+
 // position of the n-th (0-based) set bit of b (n < popc(b))
 __device__ __forceinline__ uint32_t nth_set(uint32_t b, uint32_t n) {
   uint32_t p = 0;
@@ -459,20 +463,24 @@ __device__ __forceinline__ uint32_t lead_run(const FifoWs& ws, uint32_t fe, uint
   uint32_t xc = x_begin, jc = 0, wx = 0, nw = 0, mj = 0, nq = 0, paired = 0;
   bool wdone = false, mdone = nm == 0;
   // append to a lane-aligned window the positions whose bit is set in the
-  // 32-wide chunks at cur, cur + 32, ... (four chunks loaded at once); a stop
+  // 32-wide chunks at cur, cur + 32, ... (MM_LEAD_CHUNKS loaded at once); a stop
   // bit ends the stream at its position
-  auto fill = [&](uint32_t& win, uint32_t& n, uint32_t& cur, bool& done, uint32_t lim, auto pred) {
+  auto fill = [&](uint32_t& win, uint32_t& n, uint32_t& cur, bool& done, uint32_t lim, auto load, auto pred) {
     while (!done && n < 32) {
-      uint32_t bs[4], ss[4];
+      // every chunk's loads issued before any is tested (one latency a pass)
+      uint64_t raw[MM_LEAD_CHUNKS];
 #pragma unroll
-      for (int u = 0; u < 4; u++) {
+      for (int u = 0; u < MM_LEAD_CHUNKS; u++) raw[u] = load(cur + 32 * u + lane);
+      uint32_t bs[MM_LEAD_CHUNKS], ss[MM_LEAD_CHUNKS];
+#pragma unroll
+      for (int u = 0; u < MM_LEAD_CHUNKS; u++) {
         bool in, stop;
-        pred(cur + 32 * u + lane, in, stop);
+        pred(cur + 32 * u + lane, raw[u], in, stop);
         bs[u] = __ballot_sync(kFull, in);
         ss[u] = __ballot_sync(kFull, stop);
       }
 #pragma unroll
-      for (int u = 0; u < 4; u++) {
+      for (int u = 0; u < MM_LEAD_CHUNKS; u++) {
         if (done || n >= 32) break;
         const uint32_t base = cur;
         uint32_t b = bs[u];
@@ -494,16 +502,22 @@ __device__ __forceinline__ uint32_t lead_run(const FifoWs& ws, uint32_t fe, uint
     }
   };
   while (true) {
-    fill(wx, nw, xc, wdone, W, [&](uint32_t x, bool& in, bool& stop) {
-      const bool g = x < W && ws.w_grp[x] == gg;
-      const bool run = g && ws.wl[x] < fe;
-      in = run;
-      stop = g && !run;
-    });
-    fill(mj, nq, jc, mdone, nm, [&](uint32_t j, bool& in, bool& stop) {
-      in = j < nm && (mhdr(j) & gmsk) == gh;
-      stop = false;
-    });
+    fill(
+        wx, nw, xc, wdone, W,
+        [&](uint32_t x) -> uint64_t {
+          return x < W ? ((uint64_t)ws.w_grp[x] << 16) | ws.wl[x] : ((uint64_t)kNone << 16);
+        },
+        [&](uint32_t x, uint64_t v, bool& in, bool& stop) {
+          const bool g = (uint32_t)(v >> 16) == gg;
+          in = g && (uint32_t)(v & 0xFFFFu) < fe;
+          stop = g && !in;
+        });
+    fill(
+        mj, nq, jc, mdone, nm, [&](uint32_t j) -> uint64_t { return j < nm ? mhdr(j) : 0ull; },
+        [&](uint32_t j, uint64_t v, bool& in, bool& stop) {
+          in = j < nm && (v & gmsk) == gh;
+          stop = false;
+        });
     const uint32_t n = min(nw, nq);
     if (n == 0) break;  // the run ended, or the group's messages did
     const bool act = (uint32_t)lane < n;
