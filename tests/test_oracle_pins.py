@@ -403,3 +403,42 @@ def test_jenkins_is_a_bijection_sample():
     xs = np.random.default_rng(9).choice(1 << 32, 20000, replace=False)
     hs = {oracle.jenkins32(int(x)) for x in xs}
     assert len(hs) == len(xs)
+
+
+@pytest.mark.parametrize("seed,kind,msg_frac,p_after", [(1, "src", 1.0, 0.05), (2, "tag", 0.6, 0.2),
+                                                         (3, "src", 0.4, 0.0), (4, "tag", 1.0, 0.3)])
+def test_leading_wildcard_run_takes_group_messages_in_arrival_order(seed, kind, msg_frac, p_after):
+    """The reading behind the kernel's leading-run merge,
+    checked on the oracle: wildcards of one type posted before any exact
+    receive their group admits see no competing claim, so the r-th of them
+    takes the r-th admissible message in arrival order (§II.B
+    l.65-67: earliest unmatched message, receives in posting order), or
+    nothing once the group's messages are used up."""
+    q = synth.lead_runs(seed, n_ep=3, depth=600, lead=200, kind=kind, msg_frac=msg_frac, p_wild_after=p_after,
+                        n_src=6, n_tag=4, ragged=True)
+    mr, _ = oracle.mpi_endpoints(q)
+    src = (q.recv_hdr & 0xFFFFFFFF).astype(np.int64)
+    tag = ((q.recv_hdr >> 32) & 0xFFFF).astype(np.int64)
+    msrc = (q.msg_hdr & 0xFFFFFFFF).astype(np.int64)
+    mtag = ((q.msg_hdr >> 32) & 0xFFFF).astype(np.int64)
+    checked = 0
+    for e in range(q.n_endpoints):
+        r0, r1, m0, m1 = q.recv_off[e], q.recv_off[e + 1], q.msg_off[e], q.msg_off[e + 1]
+        wild = (src[r0:r1] == synth.ANY_SOURCE) if kind == "src" else (tag[r0:r1] == synth.ANY_TAG)
+        gkey_r = tag[r0:r1] if kind == "src" else src[r0:r1]
+        gkey_m = mtag[m0:m1] if kind == "src" else msrc[m0:m1]
+        mtuples = set(zip(msrc[m0:m1].tolist(), mtag[m0:m1].tolist()))
+        for gval in np.unique(gkey_r[wild]):
+            # first exact receive admitting one of the group's messages
+            fe = r1 - r0
+            for i in range(r1 - r0):
+                if not wild[i] and gkey_r[i] == gval and (src[r0 + i], tag[r0 + i]) in mtuples:
+                    fe = i
+                    break
+            run = [i for i in range(fe) if wild[i] and gkey_r[i] == gval]
+            gmsgs = [m0 + j for j in range(m1 - m0) if gkey_m[j] == gval]
+            for r, i in enumerate(run):
+                want = gmsgs[r] if r < len(gmsgs) else -1
+                assert mr[r0 + i] == want, (e, gval, r)
+                checked += 1
+    assert checked > 100
