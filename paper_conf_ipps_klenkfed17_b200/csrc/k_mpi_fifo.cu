@@ -542,6 +542,10 @@ __device__ __forceinline__ uint32_t lead_run(const FifoWs& ws, uint32_t fe, uint
   return paired;
 }
 
+#ifndef MM_ENUM_ONCHIP
+#define MM_ENUM_ONCHIP 0  // on-chip variant: 1 = representatives enumerated directly (A/B: 0.6 % slower there)
+#endif
+
 #ifndef MM_LEAD_MIN
 #define MM_LEAD_MIN 8  // a group's wildcards from which a leading run is looked for
 #endif
@@ -945,10 +949,22 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         MM_PHASE(10);
         // warp v serves the groups g % NW == v that still have wildcards (the
         // representatives are enumerated directly: no scan of the wildcards)
+        // (on chip, MM_ENUM_ONCHIP=0: the warps scan the wildcards for group
+        // leaders instead -- A/B switch)
         const uint32_t v = (uint32_t)(NW - 1 - warp);
-        for (uint32_t b = v; b < K; b += 32 * NW) {
-          const uint32_t g = b + (uint32_t)lane * NW;
-          const bool lead = g < K && ws.gwc[g] != 0;
+        constexpr bool kEnum = !SMEM || MM_ENUM_ONCHIP;
+        const uint32_t lim = kEnum ? K : W;
+        for (uint32_t b = kEnum ? v : 0u; b < lim; b += kEnum ? 32u * NW : 32u) {
+          uint32_t g;
+          bool lead;
+          if (kEnum) {
+            g = b + (uint32_t)lane * NW;
+            lead = g < K && ws.gwc[g] != 0;
+          } else {
+            const uint32_t x = b + lane;
+            g = x < W ? ws.w_grp[x] : kNone;
+            lead = g != kNone && g % NW == v && ws.gfirst[g] == x && ws.gwc[g] != 0;
+          }
           uint32_t leaders = __ballot_sync(kFull, lead);
           while (leaders) {
             const int l = __ffs(leaders) - 1;
