@@ -542,6 +542,10 @@ __device__ __forceinline__ uint32_t lead_run(const FifoWs& ws, uint32_t fe, uint
   return paired;
 }
 
+#ifndef MM_STAGE_WLOG
+#define MM_STAGE_WLOG 1  // deep endpoints: the claim log staged in shared memory when it fits
+#endif
+
 #ifndef MM_ENUM_ONCHIP
 #define MM_ENUM_ONCHIP 0  // on-chip variant: 1 = representatives enumerated directly (A/B: 0.6 % slower there)
 #endif
@@ -575,6 +579,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     ws.rby_key = reinterpret_cast<uint16_t*>(smem_raw + L.st_rby_key);
     ws.wl = reinterpret_cast<uint16_t*>(smem_raw + L.st_wl);
     ws.recv_key = reinterpret_cast<uint16_t*>(smem_raw + L.st_recv_key);
+    if (L.st_wlog >= 0) ws.wlog = reinterpret_cast<uint16_t*>(smem_raw + L.st_wlog);
   }
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t lt = lanemask_lt();
@@ -1195,6 +1200,12 @@ FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
       L.st_wl = sb + sr;
       L.st_recv_key = sb + 2 * sr;
       L.stage_bytes = sb + 3 * sr;
+#if MM_STAGE_WLOG
+      if (L.wlog != L.msg_key && 2 * sb + 3 * sr <= kFifoStageMax) {  // P8's claim searches
+        L.st_wlog = sb + 3 * sr;
+        L.stage_bytes = 2 * sb + 3 * sr;
+      }
+#endif
     }
   }
   return L;
