@@ -1,8 +1,7 @@
+# A/B of MM_DEEP_THREADS on configs[4] (mpi_worst level), alternating builds
 cd $GRAFT_REPO_ROOT
-F=paper_conf_ipps_klenkfed17_b200/csrc/k_mpi_fifo.cu
-for t in 512 1024; do
-  sed -i "s/^#define MM_DEEP_THREADS [0-9]*/#define MM_DEEP_THREADS $t/" $F
-  python -c "from paper_conf_ipps_klenkfed17_b200 import _build; _build.build_library(force=True)" > /dev/null 2>&1
-  grep -A2 "k_mpi_fifoILi${t}ELb0" paper_conf_ipps_klenkfed17_b200/lib/ptxas.log | grep spill | head -1
-  echo "threads $t: $(python tools/config4_time.py 2>&1 | tail -1)"
-done
+for t in 512 1024; do MM_AB_DEFINES="MM_DEEP_THREADS=$t" python -c "from paper_conf_ipps_klenkfed17_b200 import _build; _build.build_library(variant='deep$t')" > /dev/null 2>&1; done
+for r in 1 2; do for t in 512 1024; do
+MM_LIB=$GRAFT_REPO_ROOT/paper_conf_ipps_klenkfed17_b200/lib/libmm_deep$t.so timeout 300 python bench.py --levels mpi_worst --no-cpu-baseline 2>/dev/null | tail -1 | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); v=d['levels']['mpi_worst']; print('threads $t', round(v['value']/1e6,2), 'M/s', round(v['roofline']['kernel_ms'],4))"
+done; done
