@@ -457,15 +457,20 @@ __device__ __forceinline__ uint32_t nth_set(uint32_t b, uint32_t n) {
 template <class MsgHdrF>
 __device__ __forceinline__ uint32_t lead_run(const FifoWs& ws, uint32_t fe, uint32_t x_begin, uint32_t W,
                                              uint32_t nm, uint32_t gg, uint64_t gmsk, MsgHdrF mhdr, int lane,
-                                             uint32_t& x_next) {
+                                             uint16_t* ring, uint32_t& x_next) {
   const uint32_t lt = lanemask_lt();
   const uint64_t gh = ws.keyhdr[gg] & gmsk;
-  uint32_t xc = x_begin, jc = 0, wx = 0, nw = 0, mj = 0, nq = 0, paired = 0;
+  // the two windows are rings of 64 positions in shared memory (this warp's
+  // ring[0..63]: wildcards, ring[64..127]: messages); at most 32 live each
+  uint16_t* wring = ring;
+  uint16_t* mring = ring + 64;
+  uint32_t xc = x_begin, jc = 0, wh = 0, nw = 0, mh = 0, nq = 0, paired = 0;
   bool wdone = false, mdone = nm == 0;
-  // append to a lane-aligned window the positions whose bit is set in the
-  // 32-wide chunks at cur, cur + 32, ... (MM_LEAD_CHUNKS loaded at once); a stop
-  // bit ends the stream at its position
-  auto fill = [&](uint32_t& win, uint32_t& n, uint32_t& cur, bool& done, uint32_t lim, auto load, auto pred) {
+  // append to a window the positions whose bit is set in the 32-wide chunks
+  // at cur, cur + 32, ... (MM_LEAD_CHUNKS loaded at once); a stop bit ends
+  // the stream at its position
+  auto fill = [&](uint16_t* rg, uint32_t h, uint32_t& n, uint32_t& cur, bool& done, uint32_t lim, auto load,
+                  auto pred) {
     while (!done && n < 32) {
       // every chunk's loads issued before any is tested (one latency a pass)
       uint64_t raw[MM_LEAD_CHUNKS];
@@ -487,7 +492,8 @@ __device__ __forceinline__ uint32_t lead_run(const FifoWs& ws, uint32_t fe, uint
         const uint32_t stop = ss[u];
         if (stop) b &= (stop & (0u - stop)) - 1u;  // the bits below the first stop
         const uint32_t nb = __popc(b), take = min(nb, 32u - n);
-        if ((uint32_t)lane >= n && (uint32_t)lane < n + take) win = base + nth_set(b, (uint32_t)lane - n);
+        const uint32_t r = __popc(b & lt);
+        if (((b >> lane) & 1u) && r < take) rg[(h + n + r) & 63u] = (uint16_t)(base + lane);
         n += take;
         if (take < nb) {
           cur = base + nth_set(b, take - 1) + 1;  // window full
@@ -503,7 +509,7 @@ __device__ __forceinline__ uint32_t lead_run(const FifoWs& ws, uint32_t fe, uint
   };
   while (true) {
     fill(
-        wx, nw, xc, wdone, W,
+        wring, wh, nw, xc, wdone, W,
         [&](uint32_t x) -> uint64_t {
           return x < W ? ((uint64_t)ws.w_grp[x] << 16) | ws.wl[x] : ((uint64_t)kNone << 16);
         },
@@ -513,14 +519,17 @@ __device__ __forceinline__ uint32_t lead_run(const FifoWs& ws, uint32_t fe, uint
           stop = g && !in;
         });
     fill(
-        mj, nq, jc, mdone, nm, [&](uint32_t j) -> uint64_t { return j < nm ? mhdr(j) : 0ull; },
+        mring, mh, nq, jc, mdone, nm, [&](uint32_t j) -> uint64_t { return j < nm ? mhdr(j) : 0ull; },
         [&](uint32_t j, uint64_t v, bool& in, bool& stop) {
           in = j < nm && (v & gmsk) == gh;
           stop = false;
         });
+    __syncwarp();  // window appends visible
     const uint32_t n = min(nw, nq);
     if (n == 0) break;  // the run ended, or the group's messages did
     const bool act = (uint32_t)lane < n;
+    const uint32_t wx = act ? wring[(wh + lane) & 63u] : 0u;
+    const uint32_t mj = act ? mring[(mh + lane) & 63u] : 0u;
     const uint32_t k = act ? (uint32_t)ws.msg_key[mj] : 0xFFFFFFFFu;
     const uint32_t peers = __match_any_sync(kFull, k);
     const uint32_t c0 = act ? (uint32_t)ws.key_c[k] : 0u;
@@ -533,12 +542,12 @@ __device__ __forceinline__ uint32_t lead_run(const FifoWs& ws, uint32_t fe, uint
     }
     __syncwarp();
     paired += n;
-    wx = __shfl_down_sync(kFull, wx, n & 31u);
-    mj = __shfl_down_sync(kFull, mj, n & 31u);
+    wh += n;
+    mh += n;
     nw -= n;
     nq -= n;
   }
-  x_next = nw ? __shfl_sync(kFull, wx, 0) : xc;
+  x_next = nw ? (uint32_t)wring[wh & 63u] : xc;
   return paired;
 }
 
@@ -566,6 +575,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
   extern __shared__ __align__(16) uint8_t smem_raw[];
   __shared__ uint64_t scan_sm[2][NT / 32];
   __shared__ uint32_t sh_K, sh_types, sh_matched;
+  // leading-run windows (global-workspace variants only): 2 rings of 64 per warp
+  __shared__ uint16_t lead_ring[SMEM ? 1 : NT / 32][128];
   constexpr int NW = NT / 32;
   // each side of the queue is cut in QP parts, placed by one warp each in P6
   // (4 for 256 threads; 16 for the 1024-thread deep-endpoint CTAs)
@@ -996,7 +1007,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
                 fe = __reduce_min_sync(kFull, fe);
                 uint32_t xn;
                 const uint32_t np = lead_run(ws, fe, x0, W, nm, gg, gmsk, [&](uint32_t j) { return MS.hdr(j); },
-                                             lane, xn);
+                                             lane, lead_ring[SMEM ? 0 : warp], xn);
                 left -= np;
                 x0 = xn;
               }
