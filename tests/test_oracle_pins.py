@@ -356,27 +356,56 @@ def test_nowild_unordered_perfect_match_all_matched():
     assert it >= 1
 
 
-def test_nowild_unordered_collisions_are_held():
-    """Three distinct keys in a table of S=1, P=5 slots whose primaries
-    collide: one receive must be held and inserted in a later iteration
-    (§VI.C l.219), and everything still matches."""
-    keys = []
-    k = 0
-    target = None
-    while len(keys) < 3:
+def _fold(h):
+    """The 64-bit header folded to the paper's 32-bit key (reading R7)."""
+    hv = int(h)
+    return oracle.jenkins32((hv & 0xFFFFFFFF) ^ oracle.jenkins32(hv >> 32))
+
+
+def _same_primary_keys(n, P, want_sec=None, S=1):
+    """n distinct tuples whose primary slots (fold % P) coincide; with
+    want_sec, the i-th key's secondary slot (J(fold) % S) is want_sec[i]."""
+    keys, target, k = [], None, 0
+    while len(keys) < n:
         h = synth.pack(k, 1)
-        hv = int(h)
-        hh = oracle.jenkins32((hv & 0xFFFFFFFF) ^ oracle.jenkins32(hv >> 32))
-        slot = hh % 5
+        f = _fold(h)
         if target is None:
-            target = slot
-        if slot == target:
+            target = f % P
+        if f % P == target and (want_sec is None or oracle.jenkins32(f) % S == want_sec[len(keys)]):
             keys.append(h)
         k += 1
-    R = np.array(keys, dtype=np.uint64)
+    return np.array(keys, dtype=np.uint64)
+
+
+def test_nowild_unordered_collisions_are_held():
+    """PAPER.md §VI.C l.219, worked by hand.  Three receives (S = 1, P = 5,
+    reading R8) whose primary slots collide, messages in reverse order.
+    Iteration 1: R0 -> primary, R1 -> secondary (first collision), R2 held
+    (second collision); M(R2) finds neither and is deferred, M(R1) hits the
+    secondary, M(R0) the primary.  Iteration 2: R2 -> primary, M(R2) hits.
+    Exactly 2 iterations -- without the secondary table it would take 3
+    (one receive tabled per iteration)."""
+    R = _same_primary_keys(3, 5)
     M = R[::-1].copy()
     mr, mm, it = oracle.nowild_unordered(R, M, return_iterations=True)
-    assert it >= 2
+    assert it == 2
+    assert (mr >= 0).all()
+    check_unordered_valid(R, M, mr, mm)
+
+
+def test_nowild_unordered_secondary_slot_is_second_hash():
+    """Five receives (S = 2, P = 10) on one primary slot; R1 and R2 have
+    different secondary slots J(key) % 2 (reading R7), R3 and R4 then collide
+    twice.  Iteration 1 tables R0 (primary), R1 and R2 (both secondary
+    slots); messages in reverse order match R2, R1, R0 and defer M(R4),
+    M(R3).  Iteration 2 tables R3 (primary) and R4 (the freed secondary
+    slot) and both match: exactly 2 iterations.  A secondary slot taken from
+    the primary hash (key % 2, equal for all five since key % 10 is) would
+    hold R2 and need 3; no secondary table, 5."""
+    R = _same_primary_keys(5, 10, want_sec=[0, 0, 1, 0, 1], S=2)
+    M = R[::-1].copy()
+    mr, mm, it = oracle.nowild_unordered(R, M, return_iterations=True)
+    assert it == 2
     assert (mr >= 0).all()
     check_unordered_valid(R, M, mr, mm)
 
@@ -395,6 +424,18 @@ def test_nowild_unordered_bruteforce(seed):
     mr, _ = oracle.nowild_unordered(R, M)
     got = {i: int(j) for i, j in enumerate(mr) if j >= 0}
     assert got in valid and len(got) == best
+
+
+def test_jenkins32_known_answers():
+    """Known-answer vectors for the paper's hash (§VI.C l.219, ref.
+    [17]: Jenkins' 32-bit 6-shift integer hash), worked line by line from the
+    published listing outside oracle/ (tests/golden/jenkins32.json, with its
+    worksheet).  A wrong constant or shift in any of the six lines changes
+    these outputs."""
+    doc = json.load(open(os.path.join(GOLDEN, "jenkins32.json")))
+    assert len(doc["vectors"]) >= 4
+    for v in doc["vectors"]:
+        assert oracle.jenkins32(int(v["in"], 16)) == int(v["steps"][-1], 16), v["in"]
 
 
 def test_jenkins_is_a_bijection_sample():
