@@ -114,6 +114,13 @@ int mm_create(mm_engine **out, int32_t semantics, int32_t n_endpoints,
 /*
  * mm_post_recvs / mm_push_msgs -- append a batch of receive requests
  * (posting order) / arrived messages (arrival order) to the endpoints.
+ * PAPER.md §II.B l.67: a new receive request looks for a message in the
+ * Unexpected Message Queue (UMQ) first, else it is appended to the Posted
+ * Receive Queue (PRQ); an arriving message looks in the PRQ, else it joins
+ * the UMQ.  Here both are batched: the posted receives and pushed messages
+ * wait, in order, behind the residual PRQ / UMQ and are matched together by
+ * the next mm_match_batch (§V l.128 treats the UMQ and new arrivals as one
+ * queue; by DESIGN.md §2.2 this gives the event-driven result).
  *   hdr         n header words, endpoint-major (all of endpoint 0 first).
  *   cookie      n int64 user handles returned in match results (e.g. request
  *               pointer / payload slot), or NULL: the engine numbers the
@@ -125,7 +132,8 @@ int mm_create(mm_engine **out, int32_t semantics, int32_t n_endpoints,
  * the next mm_match_batch has executed (stream order).  Host buffers are
  * copied by the engine asynchronously (fully so from page-locked memory) and
  * must stay valid and unchanged until the next mm_match_batch (or
- * mm_reset) returns.  At the MPI level with host hdr AND host ep_offsets the
+ * mm_reset) returns; those calls wait for the copies out of them (not for the
+ * matching), so the caller may refill the buffers as soon as they return.  At the MPI level with host hdr AND host ep_offsets the
  * copy is deferred to mm_match_batch and issued in endpoint ranges on an
  * internal copy stream (MM_OPT_PIPELINE_CHUNKS), both queues' range k before
  * range k + 1, so that it overlaps the matching of earlier ranges.  A second
@@ -165,15 +173,18 @@ int mm_push_msgs(mm_engine *e, const uint64_t *hdr, const int64_t *cookie,
 int mm_match_batch(mm_engine *e, int64_t *out_recv_cookie, int64_t *out_msg_cookie,
                    int64_t out_capacity, int64_t *counts);
 
-/* mm_reset -- empty all queues, drop pending batches, clear error flags and
- * restart cookie sequences (asynchronous). */
+/* mm_reset -- empty all queues (the PRQ and UMQ of PAPER.md §II.B l.67),
+ * drop pending batches, clear error flags and restart cookie sequences.
+ * Asynchronous on the engine stream, except that it waits for copies still
+ * reading the caller's host input buffers of a dropped batch. */
 int mm_reset(mm_engine *e);
 
 /* mm_query -- synchronise the engine's stream and fill host int64
  * vals[MM_Q_COUNT].  Returns MM_ERR_CAPACITY if the sticky flag is set. */
 int mm_query(mm_engine *e, int64_t *vals);
 
-/* mm_destroy -- free the engine (synchronises its stream).  NULL is a no-op. */
+/* mm_destroy -- free the engine and its queues (the per-endpoint PRQ / UMQ
+ * storage of PAPER.md §II.B l.67; synchronises its stream).  NULL is a no-op. */
 int mm_destroy(mm_engine *e);
 
 /*
@@ -183,7 +194,10 @@ int mm_destroy(mm_engine *e);
  *   by == 0: owner = (hash(a) * world) >> 32, a = header word (key partition;
  *            hash = the Jenkins fold of DESIGN.md reading R7);
  *   by == 1: owner = a >> 40, a = a cookie carrying its origin rank in bits
- *            40..63 (result return trip).
+ *            40..63 (result return trip).  A cookie naming no rank in
+ *            [0, world) is placed after every owner's group and is not
+ *            counted; with host `counts` the call then returns MM_ERR_ARG
+ *            (with device counts, sum(counts) < n tells).
  *   a           n inputs (device).
  *   b           n inputs (device), or NULL: b[k] = cookie_base + k.  The
  *               sharded path passes cookie_base = (rank << 40) | sequence, so

@@ -351,18 +351,18 @@ __global__ void k_materialize(Side S, int n_ep, uint64_t* q_h, int64_t* q_c, con
     }
     const int64_t k = i - S.pend_begin(e);
     const int64_t pos = (int64_t)q_len[e] + k;
-    if (pos < S.cap) {
+    if ((int64_t)q_len[e] + S.pend_count(e) <= S.cap) {
       q_h[(int64_t)e * S.cap + pos] = S.p_hdr[i];
       q_c[(int64_t)e * S.cap + pos] = S.p_cookie ? S.p_cookie[i] : S.p_seq0 + i;
-    } else {
-      atomicOr(err, kErrCapacity);
+    } else if (k == 0) {
+      atomicOr(err, kErrCapacity);  // the endpoint's pending batch does not fit: dropped whole (mm.h)
     }
   }
 }
 __global__ void k_materialize_len(Side S, int n_ep, int32_t* q_len) {
   for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < n_ep; e += gridDim.x * blockDim.x) {
-    int64_t v = (int64_t)q_len[e] + S.pend_count(e);
-    q_len[e] = (int32_t)(v < S.cap ? v : S.cap);
+    const int64_t v = (int64_t)q_len[e] + S.pend_count(e);
+    if (v <= S.cap) q_len[e] = (int32_t)v;  // else rejected: the queue keeps its contents
   }
 }
 
@@ -421,14 +421,16 @@ cudaError_t launch_finalize(const int64_t* n_out_src, int64_t n_out_host, const 
 struct OwnerOf {
   const uint64_t* a;
   int world, by;
-  __device__ __forceinline__ uint32_t operator()(int64_t k) const {
-    if (by == 1) return (uint32_t)(a[k] >> 40);
-    return (uint32_t)(((unsigned long long)header_hash(a[k]) * (unsigned)world) >> 32);
-  }
+  // by == 1: a cookie whose origin bits name no rank goes to bucket `world`,
+  // placed after every owner's group and left out of the counts
   __device__ __forceinline__ uint32_t of_payload(int64_t, uint64_t x, uint64_t) const {
-    if (by == 1) return (uint32_t)(x >> 40);
+    if (by == 1) {
+      const uint64_t o = x >> 40;
+      return o < (uint64_t)world ? (uint32_t)o : (uint32_t)world;
+    }
     return (uint32_t)(((unsigned long long)header_hash(x) * (unsigned)world) >> 32);
   }
+  __device__ __forceinline__ uint32_t operator()(int64_t k) const { return of_payload(k, a[k], 0); }
 };
 struct MoveRoute {
   const uint64_t* a;
@@ -445,11 +447,10 @@ struct MoveRoute {
     ob[dst] = (int64_t)y;
   }
 };
-__global__ void k_route_counts(const uint32_t* hist, int64_t ntiles, int world, int64_t n, int64_t* counts) {
-  int w = threadIdx.x;
-  if (w < world) {
+__global__ void k_route_counts(const uint32_t* hist, int64_t ntiles, int world, int nb, int64_t n, int64_t* counts) {
+  for (int w = threadIdx.x; w < world; w += blockDim.x) {
     int64_t s = hist[(int64_t)w * ntiles];
-    int64_t e = w + 1 < world ? (int64_t)hist[(int64_t)(w + 1) * ntiles] : n;
+    int64_t e = w + 1 < nb ? (int64_t)hist[(int64_t)(w + 1) * ntiles] : n;
     counts[w] = e - s;
   }
 }
@@ -457,11 +458,12 @@ __global__ void k_route_counts(const uint32_t* hist, int64_t ntiles, int world, 
 cudaError_t run_route(const uint64_t* a, const int64_t* b, int64_t n, int world, int by, int64_t cookie_base, uint64_t* out_a,
                       int64_t* out_b, int64_t* counts, uint32_t* part, cudaStream_t st) {
   if (n == 0) return cudaMemsetAsync(counts, 0, sizeof(int64_t) * world, st);
-  cudaError_t err = partition_stable(OwnerOf{a, world, by}, MoveRoute{a, b, out_a, out_b, cookie_base}, n, world, part, st);
+  const int nb = by == 1 ? world + 1 : world;
+  cudaError_t err = partition_stable(OwnerOf{a, world, by}, MoveRoute{a, b, out_a, out_b, cookie_base}, n, nb, part, st);
   if (err != cudaSuccess) return err;
   int64_t nt = (n + kPartTile - 1) / kPartTile;
   count_launch();
-  k_route_counts<<<1, 256, 0, st>>>(part, nt, world, n, counts);
+  k_route_counts<<<1, 256, 0, st>>>(part, nt, world, nb, n, counts);
   return cudaGetLastError();
 }
 

@@ -89,7 +89,14 @@ __global__ void k_mpi_matrix(MpiArgs a) {
   const int64_t nr = rres + a.R.pend_count(e), nm = mres + a.M.pend_count(e);
   const int64_t obase = a.out_off[e];
   if (nr > a.R.cap || nm > a.M.cap || nm > a.msg_slots || obase + nr > a.out_cap) {
+    // rejected (mm.h): receives reported unmatched if the output holds them,
+    // queues left as they were
     if (lane == 0) atomicOr(a.err, kErrCapacity);
+    if (obase + nr <= a.out_cap)
+      for (int64_t i = lane; i < nr; i += 32) {
+        a.out_rc[obase + i] = a.R.cookie(e, i, rres, rpb);
+        a.out_mc[obase + i] = (int64_t)MM_NO_MATCH;
+      }
     return;
   }
 

@@ -605,7 +605,14 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     const int64_t nr64 = rres + a.R.pend_count(e), nm64 = mres + a.M.pend_count(e);
     const int64_t obase = a.out_off[e];
     if (nr64 > a.R.cap || nm64 > a.M.cap || obase + nr64 > a.out_cap) {
+      // the endpoint's batch is rejected (mm.h): its receives are reported
+      // unmatched when the output holds them, its queues are left as they were
       if (tid == 0) atomicOr(a.err, kErrCapacity);
+      if (obase + nr64 <= a.out_cap)
+        for (int64_t i = tid; i < nr64; i += blockDim.x) {
+          a.out_rc[obase + i] = a.R.cookie(e, i, rres, rpb);
+          a.out_mc[obase + i] = (int64_t)MM_NO_MATCH;
+        }
       continue;  // uniform across the CTA
     }
     const uint32_t nr = (uint32_t)nr64, nm = (uint32_t)nm64;

@@ -177,7 +177,22 @@ struct mm_engine {
     uint32_t over;
   }* h_small = nullptr;
   int pipeline = 0;          // MM_OPT_PIPELINE_CHUNKS (0 = auto)
+  // copies out of the caller's host input buffers still in flight: recorded
+  // after they are issued (on st by post, on cs by issue_chunks) and waited
+  // for before mm_match_batch / mm_reset return, so that the caller may
+  // refill those buffers (page-locked ones included) once the call returns
+  cudaEvent_t ev_in_st = nullptr, ev_in_cs = nullptr;
+  bool in_st = false, in_cs = false;
 };
+
+// Wait until every copy out of the caller's host input buffers has executed.
+static cudaError_t release_host_inputs(mm_engine* e) {
+  cudaError_t r = cudaSuccess;
+  if (e->in_st) r = cudaEventSynchronize(e->ev_in_st);
+  if (r == cudaSuccess && e->in_cs) r = cudaEventSynchronize(e->ev_in_cs);
+  e->in_st = e->in_cs = false;
+  return r;
+}
 
 // Range k of C covers endpoints [chunk_ep(k), chunk_ep(k + 1)).  Ranges grow
 // linearly towards the middle (weights min(j + 1, C - j)): the first range's
@@ -271,6 +286,8 @@ int mm_destroy(mm_engine* e) {
       if (q->ev[k]) cudaEventDestroy(q->ev[k]);
   }
   if (e->ev_st) cudaEventDestroy(e->ev_st);
+  if (e->ev_in_st) cudaEventDestroy(e->ev_in_st);
+  if (e->ev_in_cs) cudaEventDestroy(e->ev_in_cs);
   if (e->fs) cudaStreamSynchronize(e->fs);
   if (e->fs) cudaStreamDestroy(e->fs);
   if (e->ev_fork) cudaEventDestroy(e->ev_fork);
@@ -340,6 +357,8 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
     ok = cudaStreamCreateWithFlags(&e->cs, cudaStreamNonBlocking) == cudaSuccess &&
          cudaStreamCreateWithFlags(&e->ds, cudaStreamNonBlocking) == cudaSuccess &&
          cudaEventCreateWithFlags(&e->ev_st, cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&e->ev_in_st, cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&e->ev_in_cs, cudaEventDisableTiming) == cudaSuccess &&
          cudaMallocHost(&e->h_off, (size_t)(n_endpoints + 1) * 8) == cudaSuccess;
     for (int k = 0; ok && k < kMaxChunks; k++)
       ok = cudaEventCreateWithFlags(&e->ev_k[k], cudaEventDisableTiming) == cudaSuccess &&
@@ -419,6 +438,8 @@ static int issue_chunks(mm_engine* e, Queue** qs, int nq) {
     }
   for (int i = 0; i < nq; i++)
     if (qs[i]->pend.active && qs[i]->pend.chunks > 0) qs[i]->pend.issued = true;
+  CK(cudaEventRecord(e->ev_in_cs, e->cs));
+  e->in_cs = true;
   return MM_OK;
 }
 
@@ -508,6 +529,10 @@ static int post(mm_engine* e, Queue& q, int64_t cap, const uint64_t* hdr, const 
       }
     }
   }
+  if (n > 0 && ((off && !off_dev) || !is_device_ptr(hdr) || (cookie && !is_device_ptr(cookie)))) {
+    CK(cudaEventRecord(e->ev_in_st, e->st));
+    e->in_st = true;
+  }
   q.seq += n;
   q.pend = p;
   return MM_OK;
@@ -540,6 +565,7 @@ int mm_reset(mm_engine* e) {
     q->resid_host = 0;
     q->resid_exact = true;
   }
+  CK(release_host_inputs(e));  // the dropped batch's input copies may still be in flight
   return MM_OK;
 }
 
@@ -800,8 +826,10 @@ int mm_match_batch(mm_engine* e, int64_t* out_recv_cookie, int64_t* out_msg_cook
                    int64_t* counts) {
   if (!e || out_capacity < 0 || (out_capacity > 0 && (!out_recv_cookie || !out_msg_cookie))) return MM_ERR_ARG;
   LaunchScope ls(e);
-  if (e->sem == MM_SEM_MPI) return match_mpi(e, out_recv_cookie, out_msg_cookie, out_capacity, counts);
-  return match_flat(e, out_recv_cookie, out_msg_cookie, out_capacity, counts);
+  const int rc = e->sem == MM_SEM_MPI ? match_mpi(e, out_recv_cookie, out_msg_cookie, out_capacity, counts)
+                                      : match_flat(e, out_recv_cookie, out_msg_cookie, out_capacity, counts);
+  const cudaError_t wr = release_host_inputs(e);
+  return rc != MM_OK ? rc : (wr == cudaSuccess ? MM_OK : MM_ERR_CUDA);
 }
 
 int mm_set_option(mm_engine* e, int32_t option, int64_t value) {
@@ -879,7 +907,13 @@ int mm_route(const uint64_t* a, const int64_t* b, int64_t n, int32_t world, int3
   cudaFreeAsync(part, st);
   cudaFreeAsync(dcounts, st);
   if (err == cudaSuccess && counts_host) err = cudaStreamSynchronize(st);
-  return err == cudaSuccess ? MM_OK : MM_ERR_CUDA;
+  if (err != cudaSuccess) return MM_ERR_CUDA;
+  if (counts_host && by == 1) {  // a cookie naming no rank in [0, world) was placed after the groups
+    int64_t s = 0;
+    for (int w = 0; w < world; w++) s += counts[w];
+    if (s != n) return MM_ERR_ARG;
+  }
+  return MM_OK;
 }
 
 }  // extern "C"

@@ -83,6 +83,11 @@ class Engine:
         elif not isinstance(stream, ctypes.c_void_p):
             stream = ctypes.c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
         self.stream = stream
+        self._tstream = None  # torch view of the engine stream (record_stream of device inputs)
+        torch = _torch()
+        if torch.cuda.is_available():
+            self._tstream = (torch.cuda.ExternalStream(stream.value) if stream.value
+                             else torch.cuda.default_stream())
         h = ctypes.c_void_p()
         check(L.mm_create(ctypes.byref(h), semantics, n_endpoints, recv_capacity, msg_capacity, stream), "mm_create")
         self._h = h
@@ -103,6 +108,12 @@ class Engine:
         ep_offsets = _as_i64(ep_offsets)
         n = _len(hdr)
         check(fn(self._h, _ptr(hdr), _ptr(cookie), _ptr(ep_offsets), n), name)
+        # device inputs are read on the engine stream: tell torch's caching
+        # allocator, so that a tensor freed after match_batch returns is not
+        # reused while the engine stream may still read it
+        for t in (hdr, cookie, ep_offsets):
+            if self._tstream is not None and t is not None and not isinstance(t, np.ndarray) and t.is_cuda:
+                t.record_stream(self._tstream)
         self._keep.append((hdr, cookie, ep_offsets))
 
     def post_recvs(self, hdr, cookie=None, ep_offsets=None):
