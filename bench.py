@@ -2,7 +2,7 @@
 """bench.py -- device-timed matches/s of the batched message-matching hot path.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                    [--levels mpi,ordered,unordered]
+                    [--levels mpi,mpi_cookies,...] [--no-cpu-baseline] [--nvtx]
 
 One step = one mm_match_batch over one batch of synthetic input (posted
 receives + arrived messages already resident in HBM; mm_reset + mm_post_recvs
@@ -10,14 +10,22 @@ receives + arrived messages already resident in HBM; mm_reset + mm_post_recvs
 
 Headline `value`: the MPI-compliant level on configs[1] (4096 endpoints x
 1024-deep receive/message queues, proxy-app src/tag mix, 5% ANY_SOURCE).
-`levels` adds the relaxed levels on their own workloads (configs[2]: 16M
-pairs sort+rank; configs[3]: 32M pairs per GPU hash table, 256M at 8 GPUs).
+`levels` adds: the same with user cookies (mpi_cookies), the paper-lineage
+matrix kernel (mpi_matrix), configs[2] (ordered, 16M pairs), configs[3]
+(unordered: 32M pairs per GPU, and at N=1 the full 256M on one GPU as
+unordered_256m) and configs[4] (mpi_worst).  Every level carries its
+roofline (algorithmic bytes over the engine's device-timed kernel region,
+ncu DRAM traffic of the same launches), a CPU-oracle baseline timed on this
+box's host cores, and the paper's own rate (other hardware) as context.
 Multi-GPU (torchrun): MPI endpoints are split over ranks (weak scaling, no
 collective); the no-wildcard levels shard the tuple key space with
 mm_route + NCCL all-to-all (paper_conf_ipps_klenkfed17_b200/parallel.py).
 
+--nvtx wraps each level's timed loop in an NVTX range "mm_timed:<level>" so
+that ncu can capture exactly one step's launches (tools/gpu_round.sh).
+
 Rank 0 prints ONE JSON line.  The oracle (oracle/) is only used for the
-cpu_baseline leg and for --impl reference.
+cpu_baseline legs and for --impl reference.
 """
 from __future__ import annotations
 
@@ -36,14 +44,44 @@ sys.path.insert(0, ROOT)
 
 METRIC = "matches/sec per semantics level (device-timed) at 1/2/4/8 B200; HBM GB/s"
 WORKLOADS = {
-    "mpi_matrix": "configs[1] on the compatibility-matrix kernel (MM_MPI_KERNEL_MATRIX)",
     "mpi": "configs[1]: MPI-compliant with wildcards, 4096 endpoints x 1024-deep recv/msg queues, "
-           "proxy-app-shaped src/tag mix (10-30 peers, 1..4096 tags), 5% ANY_SOURCE",
+           "proxy-app-shaped src/tag mix (10-30 peers, 1..4096 tags), 5% ANY_SOURCE; NULL cookies",
+    "mpi_cookies": "configs[1] with user cookies (a request handle per receive and per message, read by the kernel)",
+    "mpi_matrix": "configs[1] on the compatibility-matrix kernel (MM_MPI_KERNEL_MATRIX)",
     "ordered": "configs[2]: no wildcards, per-(src,tag) ordering kept: 16M recv/msg pairs via sort+rank pairing",
-    "unordered": "configs[3]: no wildcards, no ordering: 32M pairs per GPU (256M at 8 GPUs) via hash-table matching",
+    "unordered": "configs[3] per GPU: no wildcards, no ordering: 32M pairs per GPU (256M at 8 GPUs) via "
+                 "hash-table matching",
+    "unordered_256m": "configs[3] at its named size on one GPU: 256M recv/msg pairs in one engine",
     "mpi_worst": "configs[4]: worst-case MPI-compliant, one endpoint with 16K-deep queues, ANY_SOURCE receives leading "
-                 "(long match chains); L2 flushed between steps, value from the kernel region's device time",
+                 "(long match chains); L2 flushed between steps",
 }
+# The kernels inside the engine's device-timed region (roofline.kernel) and
+# the other launches of a step.
+REGION_KERNELS = {
+    "mpi": "k_mpi_fifo",
+    "mpi_cookies": "k_mpi_fifo",
+    "mpi_matrix": "k_mpi_matrix",
+    "ordered": "k_part_hist + k_scan_* + k_part_scatter (both sides, 2 passes) + k_bucket_bounds + k_bucket_pair",
+    "unordered": "k_part_hist + k_scan_* + k_part_scatter (both sides, 2 passes) + k_bucket_bounds + k_bucket_pop",
+    "unordered_256m": "k_part_hist + k_scan_* + k_part_scatter (both sides) + k_bucket_bounds + k_bucket_pop",
+    "mpi_worst": "k_mpi_fifo (1024-thread deep-endpoint instantiation, one CTA)",
+}
+# PAPER.md's own rates (GTX1080 unless stated; other hardware: context, not target)
+PAPER_CONTEXT = {
+    "mpi": "PAPER.md §V.B l.179: ~3M (Kepler), ~3.5M (Maxwell M40), ~6M (Pascal GTX1080) matches/s for the "
+           "MPI-compliant matrix algorithm, single CTA, queues <= 1024; Table II l.276/l.286: MPI <6M / ~6M "
+           "matches/s (GTX1080). CPU MPI libraries: 30M matches/s on short queues, <5M beyond 512 entries "
+           "(l.82)",
+    "ordered": "PAPER.md Table II l.296/l.306: no wildcards, ordering kept, partitioned: <60M (with unexpected "
+               "messages, compaction) / ~60M matches/s (GTX1080)",
+    "unordered": "PAPER.md §VI.C l.221: 110M (Kepler, 1 CTA, 1024 elements), 150M (Kepler, 32 CTAs), ~500M "
+                 "matches/s (Pascal GTX1080) with the two-level hash table; Table II l.316/l.326: <500M / ~500M "
+                 "(GTX1080)",
+    "mpi_worst": "PAPER.md §V.B l.181: queues above 1024 elements need several iterations and a reversed "
+                 "queue lowers the rate below the ~6M matches/s (GTX1080) of l.179",
+}
+PAPER_CONTEXT["mpi_cookies"] = PAPER_CONTEXT["mpi_matrix"] = PAPER_CONTEXT["mpi"]
+PAPER_CONTEXT["unordered_256m"] = PAPER_CONTEXT["unordered"]
 
 
 def coll_device():
@@ -77,6 +115,17 @@ def load_traffic(kernel, key="dram_bytes_per_launch"):
         d = json.load(f)
     v = d.get(kernel)
     return v.get(key) if isinstance(v, dict) else None
+
+
+def load_level_traffic(level):
+    """ncu DRAM bytes of one step's launches inside the engine's timed region
+    (NVTX range "mm_region", captured by tools/gpu_round.sh, summarised by
+    tools/level_traffic.py into profiles/level_traffic.json)."""
+    p = os.path.join(ROOT, "profiles", "level_traffic.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        return json.load(f).get(level)
 
 
 def issue_efficiency(kernel, kernel_ms, sm_mhz, sms_used=None):
@@ -156,15 +205,15 @@ def mpi_workload(rank):
     return synth.proxy_endpoints(seed=1 + 1000 * rank)
 
 
-def ordered_workload(rank, world):
+def ordered_workload(rank, world, n=None):
     import synth
-    n = (1 << 24) // world  # configs[2]: 16M pairs in total
+    n = n or (1 << 24) // world  # configs[2]: 16M pairs in total
     return synth.nowild_pairs(seed=2 + 1000 * rank, n=n, n_src=1 << 16, n_tag=64)
 
 
-def unordered_workload(rank):
+def unordered_workload(rank, n=1 << 25):
     import synth
-    return synth.nowild_pairs(seed=3 + 1000 * rank, n=1 << 25, n_src=1 << 20, n_tag=1 << 12)
+    return synth.nowild_pairs(seed=3 + 1000 * rank, n=n, n_src=1 << 20, n_tag=1 << 12)
 
 
 def to_dev(a):
@@ -172,8 +221,18 @@ def to_dev(a):
     return torch.from_numpy(np.ascontiguousarray(a).view(np.int64).copy()).cuda()
 
 
+def nvtx_range(args, level):
+    """Context manager: an NVTX range around a level's timed loop (--nvtx)."""
+    import contextlib
+
+    import torch
+    if not args.nvtx:
+        return contextlib.nullcontext()
+    return torch.cuda.nvtx.range("mm_timed:" + level)
+
+
 # --------------------------------------------------------------- our levels
-def bench_mpi(args, world, rank, peak, kernel=2, level="mpi"):
+def bench_mpi(args, world, rank, peak, kernel=2, level="mpi", cookies=False):
     import torch
 
     import paper_conf_ipps_klenkfed17_b200 as mm
@@ -185,6 +244,11 @@ def bench_mpi(args, world, rank, peak, kernel=2, level="mpi"):
     rh = [to_dev(q.recv_hdr) for _ in range(ncopy)]
     mh = [to_dev(q.msg_hdr) for _ in range(ncopy)]
     ro, mo = to_dev(q.recv_off), to_dev(q.msg_off)
+    rck = mck = [None] * ncopy
+    if cookies:  # user request handles: arbitrary 64-bit values the kernel reads and returns
+        g = torch.Generator(device="cuda").manual_seed(11)
+        rck = [torch.randint(0, 1 << 62, (n_r,), device="cuda", generator=g) for _ in range(ncopy)]
+        mck = [torch.randint(0, 1 << 62, (n_m,), device="cuda", generator=g) for _ in range(ncopy)]
     orc = [torch.empty(n_r, dtype=torch.int64, device="cuda") for _ in range(ncopy)]
     omc = [torch.empty(n_r, dtype=torch.int64, device="cuda") for _ in range(ncopy)]
     cnt = [torch.zeros(2, dtype=torch.int64, device="cuda") for _ in range(ncopy)]
@@ -193,18 +257,19 @@ def bench_mpi(args, world, rank, peak, kernel=2, level="mpi"):
     def step(i):
         s = i % ncopy
         eng.reset()
-        eng.post_recvs(rh[s], None, ro)
-        eng.push_msgs(mh[s], None, mo)
+        eng.post_recvs(rh[s], rck[s], ro)
+        eng.push_msgs(mh[s], mck[s], mo)
         eng.match_batch(orc[s], omc[s], cnt[s])
 
-    res = timed(args, step, eng, world)
+    res = timed(args, step, eng, world, level=level)
     matches = int(cnt[0][1].item())
     assert all(int(c[1].item()) == matches for c in cnt)
     q1 = eng.query()
     resid = q1["resid_recv"] + q1["resid_msg"]
     # algorithmic bytes of the matcher kernel per launch: every header read
-    # once, (recv cookie, msg cookie) written per receive, survivors compacted
-    algo = 8 * (n_r + n_m) + 16 * n_r + 16 * resid
+    # once (+ every cookie with user cookies), (recv cookie, msg cookie)
+    # written per receive, survivors compacted (header + cookie)
+    algo = 8 * (n_r + n_m) + 16 * n_r + 16 * resid + (8 * (n_r + n_m) if cookies else 0)
     res.update(matches_per_step=matches, algo_bytes=algo, n_recv=n_r, n_msg=n_m,
                kernel="k_mpi_fifo" if kernel == 2 else "k_mpi_matrix")
     if level == "mpi":
@@ -231,7 +296,7 @@ def bench_mpi_e2e(args, q, eng, world):
         eng.push_msgs(mh, None, mo)
         eng.match_batch(orc, omc, cnt)
 
-    r = timed(args, step, eng, world, query=False)
+    r = timed(args, step, eng, world, query=False, level="mpi_e2e")
     matches = int(cnt[1])
     h2d = 8 * (len(q.recv_hdr) + len(q.msg_hdr)) + 8 * (len(q.recv_off) + len(q.msg_off))
     d2h = 16 * n_r + 16
@@ -242,8 +307,9 @@ def bench_mpi_e2e(args, q, eng, world):
 
 def bench_mpi_worst(args, world, rank, peak):
     """configs[4]: one deep endpoint (per rank).  Its 256 KB of headers fit in
-    L2, so every step first overwrites a 256 MB buffer (outside the timed
-    kernel region); value = matches / the kernel region's CUDA-event time."""
+    L2, so every step first overwrites a 256 MB buffer; the level reports the
+    kernel region's CUDA-event time (value) and the step time minus the
+    separately timed flush (step_value)."""
     import torch
 
     import paper_conf_ipps_klenkfed17_b200 as mm
@@ -264,15 +330,25 @@ def bench_mpi_worst(args, world, rank, peak):
         eng.push_msgs(mh, None, mo)
         eng.match_batch(orc, omc, cnt)
 
-    res = timed(args, step, eng, world)
+    res = timed(args, step, eng, world, level="mpi_worst")
+    # the flush alone, same count, same stream
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0.record()
+    for i in range(args.steps):
+        flush.fill_(i & 0xFF)
+    e1.record()
+    torch.cuda.synchronize()
+    flush_ms = e0.elapsed_time(e1) / args.steps
     matches = int(cnt[1].item())
     # ncu counters of the 1024-thread deep-endpoint launch are keyed apart from
     # the configs[1] launch (same kernel name, different instantiation and work)
     res.update(matches_per_step=matches, algo_bytes=8 * 2 * n + 16 * n, n_recv=n, n_msg=n, kernel="k_mpi_fifo",
-               capture="k_mpi_fifo_deep", sms_used=1)
+               capture="k_mpi_fifo_deep", sms_used=1, flush_ms=flush_ms)
     eng.close()
     out = finish_level(res, world, peak, "mpi_worst")
     out["_kernel_only"] = True
+    out["_flush_ms"] = flush_ms
     return out
 
 
@@ -280,10 +356,16 @@ def bench_flat(args, world, rank, peak, level):
     import torch
 
     import paper_conf_ipps_klenkfed17_b200 as mm
-    q = ordered_workload(rank, world) if level == "ordered" else unordered_workload(rank)
+    if level == "ordered":
+        q = ordered_workload(rank, world)
+    elif level == "unordered_256m":
+        q = unordered_workload(rank, n=1 << 28)
+    else:
+        q = unordered_workload(rank)
     n = len(q.recv_hdr)
     sem = mm.MM_SEM_NOWILD_ORDERED if level == "ordered" else mm.MM_SEM_NOWILD_UNORDERED
     rh, mh = to_dev(q.recv_hdr), to_dev(q.msg_hdr)
+    del q
     if world == 1:
         eng = mm.Engine(sem, 1, n, n)
         orc = torch.empty(n, dtype=torch.int64, device="cuda")
@@ -296,8 +378,9 @@ def bench_flat(args, world, rank, peak, level):
             eng.push_msgs(mh)
             eng.match_batch(orc, omc, cnt)
 
-        res = timed(args, step, eng, world)
+        res = timed(args, step, eng, world, level=level)
         matches = int(cnt[1].item())
+        eng_q = eng
     else:
         from paper_conf_ipps_klenkfed17_b200 import parallel
         eng = parallel.ShardedMatcher(sem, capacity=2 * n)
@@ -305,16 +388,17 @@ def bench_flat(args, world, rank, peak, level):
         def step(i):
             eng.match(rh, mh)
 
-        res = timed(args, step, eng.engine, world)
+        res = timed(args, step, eng.engine, world, level=level)
         matches = eng.last_local_matches()
+        eng_q = eng.engine
     algo = 8 * 2 * n + 16 * n
-    res.update(matches_per_step=matches, algo_bytes=algo, n_recv=n, n_msg=n,
-               kernel="sort-and-rank kernels" if level == "ordered" else "hash insert+probe kernels")
+    res.update(matches_per_step=matches, algo_bytes=algo, n_recv=n, n_msg=n, kernel=REGION_KERNELS[level],
+               fallbacks=eng_q.query()["fallbacks"])
     eng.close()
     return finish_level(res, world, peak, level)
 
 
-def timed(args, step, eng, world, query=True):
+def timed(args, step, eng, world, query=True, level=""):
     import torch
     import torch.distributed as dist
     for i in range(args.warmup):
@@ -326,10 +410,11 @@ def timed(args, step, eng, world, query=True):
     torch.cuda.synchronize()
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
-    e0.record()
-    for i in range(args.steps):
-        step(args.warmup + i)
-    e1.record()
+    with nvtx_range(args, level):
+        e0.record()
+        for i in range(args.steps):
+            step(args.warmup + i)
+        e1.record()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -356,21 +441,28 @@ def finish_level(res, world, peak, level):
         t = torch.tensor([matches], dtype=torch.int64, device=coll_device())
         dist.all_reduce(t)
         total = int(t.item())
-    steps = res["steps"] if "steps" in res else None
-    del steps
     kernel_ms = res.get("kernel_ms")
     achieved = res["algo_bytes"] / (kernel_ms / 1e3) / 1e9 if kernel_ms else None
+    lt = load_level_traffic(level)
+    traffic = lt["region_dram_bytes_per_step"] if lt else None
     out = {
         "value": None, "unit": "matches/s", "workload": WORKLOADS[level],
         "matches_per_step": total, "ms_per_step": None,
         "roofline": {"bound": "hbm", "kernel": res["kernel"], "achieved": achieved, "peak": peak[0],
                      "peak_source": peak[1], "unit": "GB/s",
                      "frac": (achieved / peak[0]) if achieved else None,
-                     "traffic": load_traffic(res.get("capture", res["kernel"])),
+                     "traffic": traffic,
+                     "traffic_source": ("ncu dram__bytes_read.sum + dram__bytes_write.sum summed over the %d "
+                                        "launches of one step inside the engine's timed region (%s)"
+                                        % (lt["region_launches_per_step"], lt["source"])) if lt else None,
+                     "traffic_kernels": lt["region_kernels"] if lt else None,
                      "kernel_ms": kernel_ms, "algo_bytes_per_launch": res["algo_bytes"]},
+        "paper_context": PAPER_CONTEXT.get(level),
         "_t_ms": res["t_ms"], "_launches": res.get("launches"), "_capture": res.get("capture", res["kernel"]),
         "_sms_used": res.get("sms_used"),
     }
+    if "fallbacks" in res:
+        out["bucket_fallbacks"] = res["fallbacks"]
     if "e2e" in res:
         out["e2e"] = res["e2e"]
     return out
@@ -381,58 +473,183 @@ def finalize_values(levels, steps):
         lv["ms_per_step"] = lv["_t_ms"] / steps
         lv["value"] = lv["matches_per_step"] * steps / (lv["_t_ms"] / 1e3)
         if lv.get("_kernel_only") and lv["roofline"]["kernel_ms"]:
-            # the step also flushes L2: the level's time is its kernel region
+            # the step also flushes L2: value = the kernel region; the step
+            # minus the separately timed flush is reported beside it
+            step_ms = lv["ms_per_step"] - lv["_flush_ms"]
+            lv["step_minus_flush_ms"] = step_ms
+            lv["step_value"] = lv["matches_per_step"] / (step_ms / 1e3)
+            lv["flush_ms"] = lv["_flush_ms"]
             lv["value"] = lv["matches_per_step"] / (lv["roofline"]["kernel_ms"] / 1e3)
+            lv["value_basis"] = "kernel region (CUDA events on the engine stream); step_value: step minus L2 flush"
 
 
-# ------------------------------------------------------------ CPU baseline
-def cpu_baseline(target_s=10.0):
-    """The oracle as it stands (single-threaded C, gcc -O2) on a bounded sample
-    of the configs[1] workload (whole endpoints)."""
+# ------------------------------------------------------------ CPU baselines
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+_WORK = {}
+
+
+def _work(i):
+    """Worker body (forked process): the oracle on part i of _WORK; returns
+    (matches, seconds of oracle time)."""
+    fn, parts = _WORK["fn"], _WORK["parts"]
+    t0 = time.perf_counter()
+    n = fn(parts[i])
+    return n, time.perf_counter() - t0
+
+
+def _parallel(fn, parts):
+    """Run fn over parts in forked worker processes, one per part (the oracle
+    is plain single-threaded C with some static state, so processes, not
+    threads).  The inputs reach the workers through fork; the timed wall
+    region is the map over an already started, warmed-up pool.  Returns
+    (total matches, wall seconds)."""
+    import multiprocessing as mp
+    _WORK["fn"], _WORK["parts"] = fn, parts
+    ctx = mp.get_context("fork")
+    with ctx.Pool(len(parts)) as pool:
+        pool.map(time.sleep, [0.0] * len(parts))
+        t0 = time.perf_counter()
+        res = pool.map(_work, range(len(parts)), chunksize=1)
+        dt = time.perf_counter() - t0
+    _WORK.clear()
+    return int(sum(r[0] for r in res)), dt
+
+
+def _mpi_matches(sub):
+    import oracle
+    return int((oracle.mpi_endpoints(sub)[0] >= 0).sum())
+
+
+def _ordered_matches(p):
+    import oracle
+    return int((oracle.nowild_ordered(p[0], p[1])[0] >= 0).sum())
+
+
+def _unordered_matches(p):
+    import oracle
+    return int((oracle.nowild_unordered(p[0], p[1])[0] >= 0).sum())
+
+
+def cpu_baseline_mpi(target_s=5.0):
+    """The oracle as it stands (oracle_mpi_endpoints: the classic PRQ/UMQ
+    list traversal, plain C, gcc -O2) on a bounded sample of the configs[1]
+    workload: whole endpoints, endpoint-parallel on every host core (the
+    endpoints are independent), one process per core."""
     import oracle
     q = mpi_workload(0)
     oracle.lib()
-    n_ep = 32
+    cores = host_cores()
+    n_ep = min(q.n_endpoints, 4 * cores)
     while True:
-        sub = q.subset(range(n_ep))
-        t0 = time.perf_counter()
-        mr, _ = oracle.mpi_endpoints(sub)
-        dt = time.perf_counter() - t0
+        parts = [q.subset(range(c, n_ep, cores)) for c in range(cores)]
+        matches, dt = _parallel(_mpi_matches, parts)
         if dt * 2 >= target_s or n_ep >= q.n_endpoints:
             break
         n_ep = min(q.n_endpoints, int(n_ep * max(2.0, target_s / max(dt, 1e-3) * 0.6)))
+    return {"value": matches / dt, "unit": "matches/s", "cores": cores, "kind": "oracle",
+            "sample": "%d of 4096 configs[1] endpoints (%d matches) in %.2f s wall, oracle_mpi_endpoints "
+                      "(classic PRQ/UMQ list traversal), endpoint-parallel on %d host processes"
+                      % (n_ep, matches, dt, cores)}
+
+
+def cpu_baseline_flat(level, target_s=5.0):
+    """The no-wildcard oracles (oracle_nowild_ordered: per-source queues
+    traversed as lists; oracle_nowild_unordered: the paper's two-level hash
+    table) on the level's recipe at n pairs, n doubled until the run takes
+    a few seconds (at most the level's own size).  The tuple key space
+    partitions (§VI.A l.196), so the sample is split by tuple
+    (header % cores) and the parts run on every host core."""
+    import oracle
+    oracle.lib()
+    cores = host_cores()
+    n_max = (1 << 24) if level == "ordered" else (1 << 25)
+    n = 1 << 20
+    while True:
+        q = ordered_workload(0, 1, n=n) if level == "ordered" else unordered_workload(0, n=n)
+        kr = (q.recv_hdr % np.uint64(cores)).astype(np.int64)
+        km = (q.msg_hdr % np.uint64(cores)).astype(np.int64)
+        parts = [(q.recv_hdr[kr == c], q.msg_hdr[km == c]) for c in range(cores)]
+        matches, dt = _parallel(_ordered_matches if level == "ordered" else _unordered_matches, parts)
+        if dt * 2 >= target_s or n >= n_max:
+            break
+        n = min(n_max, n * 4)
+    name = "oracle_nowild_ordered" if level == "ordered" else "oracle_nowild_unordered (two-level hash table)"
+    return {"value": matches / dt, "unit": "matches/s", "cores": cores, "kind": "oracle",
+            "sample": "the %s recipe at %d pairs (%d matches) in %.2f s wall, %s, split by tuple over %d host "
+                      "processes" % (level, n, matches, dt, name, cores)}
+
+
+def cpu_baseline_worst():
+    """configs[4]: one endpoint, so one thread (the oracle traverses one
+    endpoint's lists sequentially)."""
+    import oracle
+    import synth
+    q = synth.worst_chain(seed=4)
+    oracle.lib()
+    t0 = time.perf_counter()
+    mr, _ = oracle.mpi_endpoints(q)
+    dt = time.perf_counter() - t0
     matches = int((mr >= 0).sum())
     return {"value": matches / dt, "unit": "matches/s", "cores": 1, "kind": "oracle",
-            "sample": "%d of 4096 configs[1] endpoints (%d matches) in %.2f s, oracle_mpi_endpoints "
-                      "(classic PRQ/UMQ list traversal, 1 thread)" % (n_ep, matches, dt)}
+            "sample": "the whole configs[4] endpoint (%d matches) in %.2f s, oracle_mpi_endpoints, 1 thread "
+                      "(a single endpoint does not split)" % (matches, dt)}
+
+
+def cpu_baselines(levels):
+    out = {}
+    if any(k in levels for k in ("mpi", "mpi_cookies", "mpi_matrix")):
+        b = cpu_baseline_mpi()
+        for k in ("mpi", "mpi_cookies", "mpi_matrix"):
+            if k in levels:
+                levels[k]["cpu_baseline"] = b
+        out["mpi"] = b
+    if "ordered" in levels:
+        levels["ordered"]["cpu_baseline"] = out["ordered"] = cpu_baseline_flat("ordered")
+    if "unordered" in levels or "unordered_256m" in levels:
+        b = cpu_baseline_flat("unordered")
+        for k in ("unordered", "unordered_256m"):
+            if k in levels:
+                levels[k]["cpu_baseline"] = b
+        out["unordered"] = b
+    if "mpi_worst" in levels:
+        levels["mpi_worst"]["cpu_baseline"] = out["mpi_worst"] = cpu_baseline_worst()
+    return out
 
 
 def run_reference(args, world, rank):
     """--impl reference: the CPU oracle, as it stands, on a bounded sample of
-    the headline workload per step (rank 0 only)."""
+    the headline workload per step, endpoint-parallel on the host cores
+    (rank 0 only)."""
     if rank != 0:
         return
     import oracle
     q = mpi_workload(0)
     oracle.lib()
-    sub = q.subset(range(64))
+    cores = host_cores()
+    n_ep = min(q.n_endpoints, 64 * cores)
+    parts = [q.subset(range(c, n_ep, cores)) for c in range(cores)]
     times, matches = [], 0
     for i in range(args.warmup + args.steps):
-        t0 = time.perf_counter()
-        mr, _ = oracle.mpi_endpoints(sub)
-        dt = time.perf_counter() - t0
+        m, dt = _parallel(_mpi_matches, parts)
         if i >= args.warmup:
             times.append(dt)
-            matches = int((mr >= 0).sum())
+            matches = m
     t = sum(times)
     v = matches * args.steps / t
+    sample = "%d of 4096 configs[1] endpoints per step, oracle_mpi_endpoints, endpoint-parallel on %d host " \
+             "processes" % (n_ep, cores)
     line = {
         "impl": "reference", "metric": METRIC, "value": v, "unit": "matches/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t / args.steps,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-        "config": {"workload": WORKLOADS["mpi"], "sample": "64 of 4096 endpoints per step"},
-        "cpu_baseline": {"value": v, "unit": "matches/s", "cores": 1, "kind": "oracle",
-                         "sample": "64 configs[1] endpoints per step, oracle_mpi_endpoints, 1 thread"},
+        "config": {"workload": WORKLOADS["mpi"], "sample": sample},
+        "cpu_baseline": {"value": v, "unit": "matches/s", "cores": cores, "kind": "oracle", "sample": sample},
         "e2e": {"value": v, "unit": "matches/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -444,8 +661,9 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--levels", default="mpi,mpi_matrix,ordered,unordered,mpi_worst")
+    ap.add_argument("--levels", default="mpi,mpi_cookies,mpi_matrix,ordered,unordered,unordered_256m,mpi_worst")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--nvtx", action="store_true", help="NVTX range per level's timed loop (ncu capture)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     world, rank, local = dist_env()
@@ -469,11 +687,15 @@ def main():
     wanted = args.levels.split(",")
     if "mpi" in wanted:
         levels["mpi"] = bench_mpi(args, world, rank, peak)
+    if "mpi_cookies" in wanted:
+        levels["mpi_cookies"] = bench_mpi(args, world, rank, peak, level="mpi_cookies", cookies=True)
     if "mpi_matrix" in wanted:
         levels["mpi_matrix"] = bench_mpi(args, world, rank, peak, kernel=1, level="mpi_matrix")
     for lv in ("ordered", "unordered"):
         if lv in wanted:
             levels[lv] = bench_flat(args, world, rank, peak, lv)
+    if "unordered_256m" in wanted and world == 1:  # N > 1: the sharded unordered level covers configs[3]
+        levels["unordered_256m"] = bench_flat(args, world, rank, peak, "unordered_256m")
     if "mpi_worst" in wanted:
         levels["mpi_worst"] = bench_mpi_worst(args, world, rank, peak)
     ck = clocks.stop()
@@ -483,6 +705,9 @@ def main():
         if rf.get("kernel", "").startswith("k_mpi"):
             lv["issue"] = issue_efficiency(lv.get("_capture", rf["kernel"]), rf.get("kernel_ms"),
                                            ck.get("sm_max_mhz") or 1965.0, lv.get("_sms_used"))
+    baselines = {}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        baselines = cpu_baselines(levels)
     head = levels.get("mpi") or next(iter(levels.values()))
     line = {
         "metric": METRIC, "value": head["value"], "unit": "matches/s", "n_gpus": world, "steps": args.steps,
@@ -490,16 +715,19 @@ def main():
         "vs_baseline": None, "dtype": "u64", "data": "synthetic",
         "config": {"workload": head["workload"], "level": "mpi" if "mpi" in levels else wanted[0],
                    "l2": "inputs > L2: 4 rotating copies of the configs[1] headers (256 MB); relaxed levels "
-                         "use 256-512 MB inputs", "parallelism": "endpoints split over %d GPU(s)" % world},
+                         "use 256 MB-4 GB inputs; configs[4] flushes L2 (256 MB write) every step",
+                   "parallelism": "endpoints split over %d GPU(s); no-wildcard levels: tuple key space sharded "
+                                  "(mm_route + all-to-all)" % world},
         "roofline": {k: v for k, v in head["roofline"].items()},
         "issue": head.get("issue"),
         "e2e": head.get("e2e"),
         "gpu_launches": head["_launches"],
         "clocks": ck,
+        "paper_context": head.get("paper_context"),
         "levels": {k: {kk: vv for kk, vv in v.items() if not kk.startswith("_")} for k, v in levels.items()},
     }
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline()
+    if baselines.get("mpi"):
+        line["cpu_baseline"] = baselines["mpi"]
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:

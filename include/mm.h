@@ -198,6 +198,12 @@ int mm_destroy(mm_engine *e);
  *            [0, world) is placed after every owner's group and is not
  *            counted; with host `counts` the call then returns MM_ERR_ARG
  *            (with device counts, sum(counts) < n tells).
+ *   by == 2: as by == 1, each owner's group split in two: first the pairs
+ *            whose b != MM_NO_MATCH, then those whose b == MM_NO_MATCH
+ *            (a = receive cookie, b = matched message cookie: the return trip
+ *            also yields each origin's matched and residual receive counts);
+ *            counts then has 2 * world entries {matched, unmatched} per
+ *            owner; b must not be NULL; world <= 255.
  *   a           n inputs (device).
  *   b           n inputs (device), or NULL: b[k] = cookie_base + k.  The
  *               sharded path passes cookie_base = (rank << 40) | sequence, so
@@ -205,7 +211,8 @@ int mm_destroy(mm_engine *e);
  *   cookie_base see b (>= 0).
  *   out_a/out_b n outputs (device), grouped by owner 0..world-1, each group in
  *               input order.
- *   counts      int64[world] (device or host) elements per owner.
+ *   counts      int64[world] (by == 2: int64[2 world]) (device or host)
+ *               elements per owner.
  *   world       1..256.
  *   stream      cudaStream_t as void*.
  * Synchronises the stream only when `counts` is host memory.

@@ -420,17 +420,27 @@ cudaError_t launch_finalize(const int64_t* n_out_src, int64_t n_out_host, const 
 // --------------------------------------------------------------- route (A6)
 struct OwnerOf {
   const uint64_t* a;
+  const int64_t* b;
   int world, by;
-  // by == 1: a cookie whose origin bits name no rank goes to bucket `world`,
-  // placed after every owner's group and left out of the counts
-  __device__ __forceinline__ uint32_t of_payload(int64_t, uint64_t x, uint64_t) const {
+  // by == 1: bucket = origin rank (bits 40..63 of the cookie a);
+  // by == 2: bucket = 2 origin + (b == MM_NO_MATCH) (results split into the
+  //          matched and the unmatched receives of each origin).
+  // A cookie whose origin bits name no rank goes to the last bucket, placed
+  // after every owner's group and left out of the counts.
+  __device__ __forceinline__ uint32_t of_payload(int64_t, uint64_t x, uint64_t y) const {
     if (by == 1) {
       const uint64_t o = x >> 40;
       return o < (uint64_t)world ? (uint32_t)o : (uint32_t)world;
     }
+    if (by == 2) {
+      const uint64_t o = x >> 40;
+      return o < (uint64_t)world ? (uint32_t)(2 * o + ((int64_t)y == (int64_t)MM_NO_MATCH)) : (uint32_t)(2 * world);
+    }
     return (uint32_t)(((unsigned long long)header_hash(x) * (unsigned)world) >> 32);
   }
-  __device__ __forceinline__ uint32_t operator()(int64_t k) const { return of_payload(k, a[k], 0); }
+  __device__ __forceinline__ uint32_t operator()(int64_t k) const {
+    return of_payload(k, a[k], by == 2 ? (uint64_t)b[k] : 0);
+  }
 };
 struct MoveRoute {
   const uint64_t* a;
@@ -457,13 +467,15 @@ __global__ void k_route_counts(const uint32_t* hist, int64_t ntiles, int world, 
 
 cudaError_t run_route(const uint64_t* a, const int64_t* b, int64_t n, int world, int by, int64_t cookie_base, uint64_t* out_a,
                       int64_t* out_b, int64_t* counts, uint32_t* part, cudaStream_t st) {
-  if (n == 0) return cudaMemsetAsync(counts, 0, sizeof(int64_t) * world, st);
-  const int nb = by == 1 ? world + 1 : world;
-  cudaError_t err = partition_stable(OwnerOf{a, world, by}, MoveRoute{a, b, out_a, out_b, cookie_base}, n, nb, part, st);
+  if (n == 0) return cudaMemsetAsync(counts, 0, sizeof(int64_t) * (by == 2 ? 2 * world : world), st);
+  const int nc = by == 2 ? 2 * world : world;  // counted buckets
+  const int nb = by == 0 ? world : nc + 1;      // + the bucket of cookies naming no rank
+  cudaError_t err =
+      partition_stable(OwnerOf{a, b, world, by}, MoveRoute{a, b, out_a, out_b, cookie_base}, n, nb, part, st);
   if (err != cudaSuccess) return err;
   int64_t nt = (n + kPartTile - 1) / kPartTile;
   count_launch();
-  k_route_counts<<<1, 256, 0, st>>>(part, nt, world, nb, n, counts);
+  k_route_counts<<<1, 256, 0, st>>>(part, nt, nc, nb, n, counts);
   return cudaGetLastError();
 }
 

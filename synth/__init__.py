@@ -26,7 +26,7 @@ ANY_TAG = 0xFFFF
 
 __all__ = [
     "ANY_SOURCE", "ANY_TAG", "pack", "Queues", "mpi_small", "mpi_endpoints",
-    "proxy_endpoints", "nowild_pairs", "worst_chain", "random_case",
+    "proxy_endpoints", "nowild_pairs", "worst_chain", "random_case", "widen",
 ]
 
 
@@ -254,3 +254,42 @@ def random_case(seed, n_ep=3, max_depth=40, wild=True, n_src=4, n_tag=4, n_comm=
     return mpi_endpoints(int(rng.integers(1 << 30)), n_ep, max_depth, n_src=n_src,
                          n_tag=n_tag, p_any_src=p, p_any_tag=p, n_comm=n_comm,
                          ragged=True, p_unmatched=0.2)
+
+
+def widen(q, seed, p_msg_any_src=0.0, p_msg_any_tag=0.0):
+    """The same queues with full-width header fields: every small source id
+    is mapped to a distinct random 32-bit value (near-ANY values such as
+    0xFFFFFFFE included), every tag to a random 16-bit value (0xFFFE
+    included), every communicator to a random 16-bit value; wildcards stay
+    wildcards.  p_msg_any_*: fraction of messages that carry the reserved
+    wildcard values themselves (matched literally, reading R2).  Only the
+    field values change, not which fields are equal."""
+    rng = np.random.default_rng(seed)
+
+    def remap(x, width, any_val):
+        u = np.unique(x[x != any_val]) if any_val is not None else np.unique(x)
+        pool = np.array([(1 << width) - 2, (1 << width) - 3, 0], dtype=np.uint64)
+        rand = rng.choice((1 << width) - 1, size=len(u) + 8, replace=False).astype(np.uint64)
+        vals = np.unique(np.concatenate([pool, rand]))
+        vals = rng.permutation(vals[vals != np.uint64((1 << width) - 1)])[:len(u)]
+        out = x.copy()
+        if len(u):
+            idx = np.searchsorted(u, x)
+            keep = (x != any_val) if any_val is not None else np.ones(len(x), bool)
+            out[keep] = vals[idx[keep]]
+        return out
+
+    def fields(h):
+        return h & np.uint64(0xFFFFFFFF), (h >> np.uint64(32)) & np.uint64(0xFFFF), h >> np.uint64(48)
+
+    rs, rt, rc = fields(q.recv_hdr)
+    ms, mt, mc = fields(q.msg_hdr)
+    nr = len(rs)
+    src = remap(np.concatenate([rs, ms]), 32, np.uint64(ANY_SOURCE))
+    tag = remap(np.concatenate([rt, mt]), 16, np.uint64(ANY_TAG))
+    comm = remap(np.concatenate([rc, mc]), 16, None)
+    msrc, mtag = src[nr:], tag[nr:]
+    msrc[rng.random(len(msrc)) < p_msg_any_src] = ANY_SOURCE
+    mtag[rng.random(len(mtag)) < p_msg_any_tag] = ANY_TAG
+    return Queues(pack(src[:nr], tag[:nr], comm[:nr]), q.recv_off, pack(msrc, mtag, comm[nr:]), q.msg_off,
+                  q.name + "[wide]")

@@ -126,3 +126,27 @@ def per_key_min_np(recv_hdr, msg_hdr):
     km, cm = np.unique(msg_hdr, return_counts=True)
     common, ia, ib = np.intersect1d(ku, km, assume_unique=True, return_indices=True)
     return common, np.minimum(cu[ia], cm[ib])
+
+
+def check_unordered_per_batch(results, batches, recv_hdr_by_cookie, msg_hdr_by_cookie):
+    """NOWILD_UNORDERED over several batches, batch by batch (reading R6):
+    the snapshot is the engine's own residual plus the batch; every snapshot
+    receive is reported once; matched pairs have equal tuples and use each
+    snapshot message at most once; every tuple gets min(#recv, #msg) of the
+    snapshot (a maximal pairing); the residuals carry over."""
+    res_r = np.zeros(0, np.int64)
+    res_m = np.zeros(0, np.int64)
+    for b, ((grc, gmc, _), (rh, rc, ro, mh, mc, mo)) in enumerate(zip(results, batches)):
+        snap_r = np.concatenate([res_r, np.asarray(rc, np.int64)])
+        snap_m = np.concatenate([res_m, np.asarray(mc, np.int64)])
+        assert np.array_equal(np.sort(grc), np.sort(snap_r)), "batch %d: snapshot receives" % b
+        m = gmc >= 0
+        used = gmc[m]
+        assert len(np.unique(used)) == len(used), "batch %d: a message matched twice" % b
+        assert np.isin(used, snap_m).all(), "batch %d: a message outside the snapshot" % b
+        assert np.array_equal(recv_hdr_by_cookie[grc[m]], msg_hdr_by_cookie[used]), "batch %d: tuples" % b
+        keys, mins = per_key_min_np(recv_hdr_by_cookie[snap_r], msg_hdr_by_cookie[snap_m])
+        got_k, got_c = np.unique(recv_hdr_by_cookie[grc[m]], return_counts=True)
+        assert np.array_equal(got_k, keys) and np.array_equal(got_c, mins), "batch %d: not maximal per tuple" % b
+        res_r = grc[~m]
+        res_m = snap_m[~np.isin(snap_m, used)]

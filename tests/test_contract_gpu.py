@@ -175,3 +175,30 @@ def test_route_cookie_naming_no_rank():
     assert np.array_equal(ob.cpu().numpy()[k:], np.nonzero(bad)[0])
     with pytest.raises(MMError):
         route(da, None, world, 1, oa, ob, np.zeros(world, np.int64))
+
+
+@pytest.mark.parametrize("world", [1, 3, 8, 255])
+def test_route_by_origin_matched_first(world):
+    """mm_route by == 2 (the sharded return trip): grouped by origin rank,
+    within each origin the matched results (b != MM_NO_MATCH) before the
+    unmatched ones, each part in input order; counts {matched, unmatched}
+    per origin; a cookie naming no rank after everything, uncounted."""
+    import torch
+    from paper_conf_ipps_klenkfed17_b200 import route
+    rng = np.random.default_rng(world)
+    n = 40000
+    owner = rng.integers(0, world, n).astype(np.uint64)
+    bad = rng.random(n) < 0.002
+    owner[bad] = np.uint64(world + 3)
+    a = (owner << np.uint64(40)) | rng.integers(0, 1 << 40, n).astype(np.uint64)
+    b = np.where(rng.random(n) < 0.3, -1, rng.integers(0, 1 << 50, n)).astype(np.int64)
+    da, db = torch.from_numpy(a.view(np.int64)).cuda(), torch.from_numpy(b).cuda()
+    oa, ob = torch.empty_like(da), torch.empty_like(db)
+    counts = torch.zeros(2 * world, dtype=torch.int64, device="cuda")
+    route(da, db, world, 2, oa, ob, counts)
+    torch.cuda.synchronize()
+    key = np.where(bad, 2 * world, 2 * owner.astype(np.int64) + (b == -1))
+    order = np.argsort(key, kind="stable")
+    assert np.array_equal(oa.cpu().numpy().view(np.uint64), a[order])
+    assert np.array_equal(ob.cpu().numpy(), b[order])
+    assert np.array_equal(counts.cpu().numpy(), np.bincount(key[~bad], minlength=2 * world))

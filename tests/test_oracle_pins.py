@@ -107,6 +107,25 @@ def test_mpi_bruteforce_unique_and_equal(seed):
     assert (mm >= 0).sum() == len(got)
 
 
+@pytest.mark.parametrize("seed", range(40))
+def test_mpi_bruteforce_wide_fields_and_literal_any(seed):
+    """As above with full-width field values (src near 2^32, tag near 2^16,
+    16-bit communicators) and messages that carry the reserved wildcard
+    values themselves (reading R2: matched literally -- only a receive whose
+    field is the wildcard admits them)."""
+    rng = np.random.default_rng(7000 + seed)
+    nr, nm = int(rng.integers(0, 5)), int(rng.integers(0, 5))
+    sv = np.array([ANY_S, 0xFFFFFFFE, 0x80000000], dtype=np.uint64)
+    tv = np.array([ANY_T, 0xFFFE, 0x8000], dtype=np.uint64)
+    cv = np.array([0xFFFF, 0x8001], dtype=np.uint64)
+    R = synth.pack(sv[rng.integers(0, 3, nr)], tv[rng.integers(0, 3, nr)], cv[rng.integers(0, 2, nr)])
+    M = synth.pack(sv[rng.integers(0, 3, nm)], tv[rng.integers(0, 3, nm)], cv[rng.integers(0, 2, nm)])
+    sols = [pi for pi in all_partial_injections(nr, nm) if mpi_rules_hold(R, M, pi)]
+    assert len(sols) == 1
+    mr, _ = oracle.mpi_two_list(R, M)
+    assert {i: int(j) for i, j in enumerate(mr) if j >= 0} == sols[0]
+
+
 def paper_algorithms_1_2(R, M, warp=4):
     """PAPER.md §V.A, executed literally.  Algorithm 1 (l.151-158): thread t
     holds message t, for every receive i a warp ballots SendObj == RecvObj and

@@ -10,7 +10,8 @@ import pytest
 
 import oracle
 import synth
-from _util import (check_unordered, gpu_batches, oracle_batches, per_key_min, per_key_min_np, single_batch,
+from _util import (check_unordered, check_unordered_per_batch, gpu_batches, oracle_batches, per_key_min, per_key_min_np,
+                   single_batch,
                    split_batches)
 
 pytestmark = pytest.mark.gpu
@@ -237,6 +238,35 @@ def test_mpi_config4_worst_chain(kern):
     assert_exact(g, o)
 
 
+@KERNELS
+@pytest.mark.parametrize("seed,p_any", [(1, 0.0), (2, 0.1), (3, 0.3)])
+def test_mpi_wide_headers_and_literal_any(kern, seed, p_any):
+    """Full-width header fields (32-bit src, 16-bit tag and comm, values next
+    to the wildcard ones) and messages carrying the reserved ANY values
+    (reading R2), ragged endpoints, both wildcard kinds, two communicators,
+    unexpected messages, 3 batches with residual queues -- bit-exact."""
+    rng = np.random.default_rng(seed)
+    q = synth.widen(synth.mpi_endpoints(seed, n_ep=40, depth_r=300, n_src=12, n_tag=6, n_comm=2, ragged=True,
+                                        p_unmatched=0.2, p_any_src=0.2, p_any_tag=0.15),
+                    seed, p_msg_any_src=p_any, p_msg_any_tag=p_any)
+    batches = split_batches(q, 3, rng)
+    g, st = gpu_batches(MPI, 40, 300, 300, batches, mpi_kernel=kern)
+    o, _ = oracle_batches(MPI, 40, batches)
+    assert_exact(g, o)
+    assert st["error"] == 0
+
+
+@pytest.mark.parametrize("kind", ["src", "tag"])
+def test_mpi_wide_headers_deep_endpoint(kind):
+    """The deep-endpoint (global workspace, 1024-thread) variant on wide
+    headers with a leading wildcard run and literal-ANY messages."""
+    q = synth.widen(synth.lead_runs(5, n_ep=1, depth=6000, lead=1500, kind=kind, n_src=20, n_tag=6),
+                    5, p_msg_any_src=0.05, p_msg_any_tag=0.05)
+    g, st = gpu_batches(MPI, 1, 6000, 6000, single_batch(q))
+    o, _ = oracle_batches(MPI, 1, single_batch(q))
+    assert_exact(g, o)
+
+
 @pytest.mark.parametrize("case", ["worst", "mixed"])
 def test_mpi_maximum_capacity(case):
     """Queues at the MPI level's maximum capacity (MM_MPI_MAX_MSGS, global
@@ -427,6 +457,7 @@ def test_unordered_multibatch(seed, flat):
     assert len(np.unique(rc[m])) == m.sum() and len(np.unique(mc[m])) == m.sum()
     assert np.array_equal(q.recv_hdr[rc[m]], q.msg_hdr[mc[m]])
     assert int(m.sum()) == check_min(q)
+    check_unordered_per_batch(g, batches, q.recv_hdr, q.msg_hdr)
 
 
 @pytest.mark.slow
@@ -441,6 +472,48 @@ def test_unordered_config3_per_gpu(flat):
     assert len(np.unique(gmc[m])) == int(m.sum())
     keys, mins = per_key_min_np(q.recv_hdr, q.msg_hdr)
     assert int(m.sum()) == int(mins.sum()) == int(cnt[1])
+
+
+@pytest.mark.slow
+def test_unordered_config3_full_256m():
+    """configs[3] at its named size on one B200: 256M receive/message pairs
+    in one engine (§VI.C l.213-221; the 8-GPU run shards the same key
+    space).  Checked on the device with torch (the properties reading R6
+    fixes at any size): every receive reported once, matched pairs carry
+    equal tuples, each message used once, and the match count equals
+    sum over tuples of min(#recv, #msg) -- with validity this forces every
+    tuple to its own min (a maximal pairing)."""
+    import torch
+    from paper_conf_ipps_klenkfed17_b200 import MM_SEM_NOWILD_UNORDERED, Engine
+    n = 1 << 28
+    q = synth.nowild_pairs(3, n=n, n_src=1 << 20, n_tag=1 << 12)
+    rh = torch.from_numpy(q.recv_hdr.view(np.int64)).cuda()
+    mh = torch.from_numpy(q.msg_hdr.view(np.int64)).cuda()
+    del q
+    eng = Engine(MM_SEM_NOWILD_UNORDERED, 1, n, n)
+    orc = torch.empty(n, dtype=torch.int64, device="cuda")
+    omc = torch.empty(n, dtype=torch.int64, device="cuda")
+    cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+    eng.post_recvs(rh)
+    eng.push_msgs(mh)
+    eng.match_batch(orc, omc, cnt)
+    st = eng.query()
+    eng.close()
+    assert st["error"] == 0
+    assert int(cnt[0]) == n
+    assert torch.equal(torch.sort(orc).values, torch.arange(n, device="cuda"))
+    m = omc >= 0
+    n_matched = int(m.sum())
+    assert n_matched == int(cnt[1])
+    assert torch.equal(rh[orc[m]], mh[omc[m]]), "matched tuples differ"
+    used = torch.sort(omc[m]).values
+    assert not bool((used[1:] == used[:-1]).any()), "a message matched twice"
+    del used, orc, omc, m
+    kr, cr = torch.unique_consecutive(torch.sort(rh).values, return_counts=True)
+    km, cm = torch.unique_consecutive(torch.sort(mh).values, return_counts=True)
+    pos = torch.searchsorted(km, kr).clamp(max=len(km) - 1)
+    hit = km[pos] == kr
+    assert n_matched == int(torch.minimum(cr[hit], cm[pos[hit]]).sum())
 
 
 # ------------------------------------------------------------------- route
