@@ -164,9 +164,7 @@ struct mm_engine {
   DBuf skey[2], sval[2], rid, run_start, run_rc, part;
   DBuf owner, rcnt, mcnt, tkey, tval;
   int64_t T = 0;
-  DBuf bh[4], bi[4], bpart, bpart2, broff, bmoff, bover;
-  cudaStream_t fs = nullptr;  // no-wildcard levels: the message side's partition stream
-  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  DBuf bh[2], bix[2], bsflag[2], bxh[2][2], bxix[2][2], bcnt, broff, bscan, bover;  // bucket regions (k_bucket.cu)
   int flat_kernel = MM_FLAT_KERNEL_BUCKETED;
   long long bucket_fallbacks = 0;
   Timer timer;
@@ -294,10 +292,6 @@ int mm_destroy(mm_engine* e) {
   if (e->ev_st) cudaEventDestroy(e->ev_st);
   if (e->ev_in_st) cudaEventDestroy(e->ev_in_st);
   if (e->ev_in_cs) cudaEventDestroy(e->ev_in_cs);
-  if (e->fs) cudaStreamSynchronize(e->fs);
-  if (e->fs) cudaStreamDestroy(e->fs);
-  if (e->ev_fork) cudaEventDestroy(e->ev_fork);
-  if (e->ev_join) cudaEventDestroy(e->ev_join);
   if (e->cs) cudaStreamDestroy(e->cs);
   if (e->ds) cudaStreamDestroy(e->ds);
   if (e->h_off) cudaFreeHost(e->h_off);
@@ -316,8 +310,9 @@ int mm_destroy(mm_engine* e) {
                   &e->out_mc_stage, &e->rflag, &e->mflag, &e->scan, &e->skey[0], &e->skey[1],
                   &e->sval[0], &e->sval[1], &e->rid, &e->run_start, &e->run_rc, &e->part,
                   &e->owner, &e->rcnt, &e->mcnt, &e->tkey, &e->tval, &e->fifo_ws,
-                  &e->bh[0], &e->bh[1], &e->bh[2], &e->bh[3], &e->bi[0], &e->bi[1], &e->bi[2], &e->bi[3],
-                  &e->bpart, &e->bpart2, &e->broff, &e->bmoff, &e->bover};
+                  &e->bh[0], &e->bh[1], &e->bix[0], &e->bix[1], &e->bsflag[0], &e->bsflag[1], &e->bcnt,
+                  &e->broff, &e->bscan, &e->bover, &e->bxh[0][0], &e->bxh[0][1], &e->bxh[1][0], &e->bxh[1][1],
+                  &e->bxix[0][0], &e->bxix[0][1], &e->bxix[1][0], &e->bxix[1][1]};
   for (DBuf* b : bufs) release(*b);
   delete e;
   return MM_OK;
@@ -382,17 +377,21 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
     const int64_t n = e->rcap + e->mcap;
     ok = ensure(e->rflag, e->rcap) == cudaSuccess && ensure(e->mflag, e->mcap) == cudaSuccess &&
          ensure(e->scan, (size_t)scan_scratch_elems(n) * 8) == cudaSuccess;
-    for (int b = 0; ok && b < 4; b++) {
-      const int64_t c = b < 2 ? e->rcap : e->mcap;
-      ok = ensure(e->bh[b], c * 8) == cudaSuccess && ensure(e->bi[b], c * 8) == cudaSuccess;
+    // bucket regions sized for the larger side (k_bucket.cu)
+    const int64_t side = e->rcap > e->mcap ? e->rcap : e->mcap;
+    const PartPlan pl = part_plan_alloc(side);
+    const int64_t nbk = bucket_count(side), slots = nbk * pl.cap[pl.passes - 1];
+    for (int b = 0; ok && b < 2; b++) {
+      ok = ensure(e->bh[b], (size_t)slots * 8) == cudaSuccess && ensure(e->bix[b], (size_t)slots * 4) == cudaSuccess &&
+           ensure(e->bsflag[b], (size_t)slots) == cudaSuccess;
+      for (int x = 0; ok && x < 2; x++)
+        if (pl.scratch_slots[x] > 0)
+          ok = ensure(e->bxh[x][b], (size_t)pl.scratch_slots[x] * 8) == cudaSuccess &&
+               ensure(e->bxix[x][b], (size_t)pl.scratch_slots[x] * 4) == cudaSuccess;
     }
-    ok = ok && ensure(e->bpart, (size_t)partition_scratch_elems(e->rcap) * 4) == cudaSuccess &&
-         ensure(e->bpart2, (size_t)partition_scratch_elems(e->mcap) * 4) == cudaSuccess &&
-         cudaStreamCreateWithFlags(&e->fs, cudaStreamNonBlocking) == cudaSuccess &&
-         cudaEventCreateWithFlags(&e->ev_fork, cudaEventDisableTiming) == cudaSuccess &&
-         cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming) == cudaSuccess &&
-         ensure(e->broff, (size_t)bucket_scratch_elems(n) * 4) == cudaSuccess &&
-         ensure(e->bmoff, (size_t)bucket_scratch_elems(n) * 4) == cudaSuccess && ensure(e->bover, 4) == cudaSuccess;
+    ok = ok && ensure(e->bcnt, (size_t)pl.cnt_total * 4) == cudaSuccess &&
+         ensure(e->broff, (size_t)(nbk + 1) * 4) == cudaSuccess &&
+         ensure(e->bscan, (size_t)scan_scratch_elems(nbk) * 4) == cudaSuccess && ensure(e->bover, 4) == cudaSuccess;
     if (ok && semantics == MM_SEM_NOWILD_ORDERED) {
       ok = ensure(e->skey[0], n * 8) == cudaSuccess && ensure(e->skey[1], n * 8) == cudaSuccess &&
            ensure(e->sval[0], n * 4) == cudaSuccess && ensure(e->sval[1], n * 4) == cudaSuccess &&
@@ -731,31 +730,30 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
   unsigned long long matched_host = 0;  // pairs of the bucketed run (valid when done)
   BucketScratch bs;
   if (e->flat_kernel == MM_FLAT_KERNEL_BUCKETED) {
-    for (int b = 0; b < 4; b++) {
+    for (int b = 0; b < 2; b++) {
       bs.h[b] = (uint64_t*)e->bh[b].p;
-      bs.i[b] = (uint64_t*)e->bi[b].p;
+      bs.ix[b] = (uint32_t*)e->bix[b].p;
+      bs.sflag[b] = (uint8_t*)e->bsflag[b].p;
+      for (int x = 0; x < 2; x++) {
+        bs.xh[x][b] = (uint64_t*)e->bxh[x][b].p;
+        bs.xix[x][b] = (uint32_t*)e->bxix[x][b].p;
+      }
     }
-    bs.part = (uint32_t*)e->bpart.p;
-    bs.part2 = (uint32_t*)e->bpart2.p;
-    bs.side_st = e->fs;
-    bs.ev_fork = e->ev_fork;
-    bs.ev_join = e->ev_join;
+    bs.cnt = (uint32_t*)e->bcnt.p;
     bs.roff = (uint32_t*)e->broff.p;
-    bs.moff = (uint32_t*)e->bmoff.p;
+    bs.scan = (uint32_t*)e->bscan.p;
     bs.overflow = (uint32_t*)e->bover.p;
     bs.rres = info.rres;
     bs.mres = info.mres;
     e->timer.begin(e->st);
     CK(run_bucketed(a, ordered, bs, e->st));
     e->timer.end(e->st);
-    uint32_t over = 0;
     CK(cudaMemcpyAsync(&e->h_small->over, e->bover.p, 4, cudaMemcpyDeviceToHost, e->st));
     CK(cudaMemcpyAsync(&e->h_small->matched, e->nmatched.p, 8, cudaMemcpyDeviceToHost, e->st));
     CK(cudaStreamSynchronize(e->st));
-    over = e->h_small->over;
     matched_host = e->h_small->matched;
-    done = over == 0;
-    if (!done) {  // a bucket exceeded the on-chip capacity (heavily repeated tuples)
+    done = e->h_small->over == 0;
+    if (!done) {  // a bucket exceeded its region or the on-chip capacity (heavily repeated tuples)
       e->bucket_fallbacks++;
       CK(cudaMemsetAsync(e->nmatched.p, 0, 8, e->st));
     }
@@ -806,13 +804,13 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
       // every element of this side matched (known from the count read back
       // with the overflow flag): the residual queue is empty, no compaction
       CK(cudaMemsetAsync(q.len[nb].p, 0, 4, e->st));
-    } else if (done)  // bucketed: flags and survivors in bucket order
-      CK(run_compact_sorted(*ss[i], res[i], ns[i], i == 0 ? bs.rh_sorted : bs.mh_sorted,
-                            i == 0 ? bs.ri_sorted : bs.mi_sorted, fl[i], (uint64_t*)q.hdr[nb].p,
-                            (int64_t*)q.cookie[nb].p, (int32_t*)q.len[nb].p, (uint32_t*)e->scan.p, e->st));
-    else
+    } else {
+      // bucketed: the slots' matched bytes to snapshot order first, so that
+      // the residual queue keeps posting / arrival order
+      if (done) CK(run_slot_flags(bs, i, (uint8_t*)fl[i], e->st));
       CK(run_compact(*ss[i], res[i], ns[i], fl[i], (uint64_t*)q.hdr[nb].p, (int64_t*)q.cookie[nb].p,
                      (int32_t*)q.len[nb].p, (uint32_t*)e->scan.p, e->st));
+    }
     q.cur = nb;
     q.pend = Pending();
     if (done) {  // each pair consumed one element of each side: the residual size is exact

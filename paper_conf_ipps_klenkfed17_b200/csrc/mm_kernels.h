@@ -94,31 +94,43 @@ struct HashScratch {
 };
 cudaError_t run_hash(const FlatArgs& a, const HashScratch& h, cudaStream_t st);
 
-// Both no-wildcard levels, hash-bucketed (k_bucket.cu): stable partition into
-// ~1K-element buckets + one CTA per bucket.  Sets *overflow if a bucket does
-// not fit on chip (the caller then falls back to run_sort_rank / run_hash).
-struct BucketScratch {
-  uint64_t* h[4];  // receive ping-pong (0,1), message ping-pong (2,3)
-  uint64_t* i[4];  // (bucket << 32) | snapshot index
-  uint32_t* part;   // partition scratch of the receive side
-  uint32_t* part2;  // ... of the message side (partitioned concurrently on side_st)
-  uint32_t* roff;
-  uint32_t* moff;
-  uint32_t* overflow;
-  cudaStream_t side_st;            // nullptr: both sides on the engine stream
-  cudaEvent_t ev_fork, ev_join;
-  int64_t rres, mres;
-  // outputs: the bucket-sorted sides (results are written in this order)
-  const uint64_t* rh_sorted;
-  const uint64_t* ri_sorted;
-  const uint64_t* mh_sorted;
-  const uint64_t* mi_sorted;
+// Both no-wildcard levels, hash-bucketed (k_bucket.cu): one-pass partition
+// into fixed-capacity bucket regions + one CTA per bucket.  Sets *overflow if
+// a bucket does not fit (the caller then falls back to run_sort_rank /
+// run_hash).
+constexpr int kMaxPasses = 4;
+struct PartPlan {                 // partition passes for a side of n_side elements (k_bucket.cu)
+  int nb, passes;
+  int bits[kMaxPasses], shift[kMaxPasses];
+  int64_t children[kMaxPasses];   // regions per side after pass i
+  int64_t cap[kMaxPasses];        // slots per region after pass i
+  int64_t slots[kMaxPasses];      // children x cap
+  int64_t cnt_off[kMaxPasses];    // offset of pass i's counts [2][children] in the count array
+  int64_t cnt_total;
+  int64_t scratch_slots[2];       // intermediate levels alternate between two buffers
 };
+PartPlan part_plan(int64_t n_side);
+PartPlan part_plan_alloc(int64_t n_side);  // the largest any batch up to n_side needs
+struct BucketScratch {
+  uint64_t* h[2];      // final bucket regions (plan.slots[last]): headers (receives, messages)
+  uint32_t* ix[2];     // ... snapshot indices
+  uint8_t* sflag[2];   // ... matched byte per slot
+  uint64_t* xh[2][2];  // intermediate regions [buffer][side]
+  uint32_t* xix[2][2];
+  uint32_t* cnt;       // every pass's region counts (plan.cnt_total)
+  uint32_t* roff;      // [B + 1] output offsets of the buckets
+  uint32_t* scan;      // scan scratch (scan_scratch_elems(B))
+  uint32_t* overflow;
+  int64_t rres, mres;
+  PartPlan plan;       // set by run_bucketed
+  const uint32_t* bcnt;  // final counts [2][B] (set by run_bucketed)
+  uint32_t B;
+};
+int bucket_bits_for(int64_t n_side);
+int64_t bucket_count(int64_t n_side);
 cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cudaStream_t st);
-cudaError_t run_compact_sorted(const Side& S, int64_t resid, int64_t n, const uint64_t* h, const uint64_t* ix,
-                               const uint8_t* matched, uint64_t* q_h, int64_t* q_c, int32_t* q_len, uint32_t* scan,
-                               cudaStream_t st);
-int64_t bucket_scratch_elems(int64_t n);
+// snapshot-order matched flags of one side from the bucket slots (partly matched sides)
+cudaError_t run_slot_flags(const BucketScratch& s, int side, uint8_t* flag, cudaStream_t st);
 
 // Compaction of the no-wildcard queues into the other ping-pong buffer.
 cudaError_t run_compact(const Side& S, int64_t resid, int64_t n, const uint8_t* matched, uint64_t* q_h, int64_t* q_c,
