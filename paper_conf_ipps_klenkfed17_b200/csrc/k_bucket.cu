@@ -69,8 +69,17 @@ int64_t bucket_count(int64_t n_side) { return (int64_t)1 << bucket_bits_for(n_si
 // snapshot index travels with the header and the matching kernel orders
 // equal tuples by it where order matters.  Reads 8 B (pass 0) or 12 B and
 // writes 12 B per element and pass.
-constexpr int kPassThreads = 512;
-constexpr int kPassItems = 8;
+#ifndef MM_PASS_THREADS
+#define MM_PASS_THREADS 512  // A/B (tools/gpu_ab_pass.sh): 512 x 8 x 2 CTAs/SM beats 256 x 8/16, 1024 x 4/8, 512 x 4/16
+#endif
+#ifndef MM_PASS_ITEMS
+#define MM_PASS_ITEMS 8
+#endif
+#ifndef MM_PASS_MINB
+#define MM_PASS_MINB 2
+#endif
+constexpr int kPassThreads = MM_PASS_THREADS;
+constexpr int kPassItems = MM_PASS_ITEMS;
 constexpr int kPassTile = kPassThreads * kPassItems;  // 4096
 constexpr int kPassMaxKeys = 1024;                    // digits per tile (pass 0: both sides' digits)
 
@@ -147,7 +156,7 @@ struct PassSmem {
 };
 
 template <bool FIRST>
-__global__ void __launch_bounds__(kPassThreads, 2) k_part_pass(PassArgs a) {
+__global__ void __launch_bounds__(kPassThreads, MM_PASS_MINB) k_part_pass(PassArgs a) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   PassSmem& sm = *reinterpret_cast<PassSmem*>(smem_raw);
   const int tid = threadIdx.x;
