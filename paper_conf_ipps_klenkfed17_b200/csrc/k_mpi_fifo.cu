@@ -559,6 +559,11 @@ __device__ __forceinline__ uint32_t lead_run(const FifoWs& ws, uint32_t fe, uint
 #define MM_ENUM_ONCHIP 0  // on-chip variant: 1 = representatives enumerated directly (A/B: 0.6 % slower there)
 #endif
 
+#ifndef MM_DP_LEAD
+#define MM_DP_LEAD 1  // leading runs resolved by CTA-wide scans (0: one warp merges each run, lead_run)
+#endif
+constexpr uint32_t kLeadList = 1024;  // groups with a leading run handled per endpoint (more: the chain serves them)
+
 #ifndef MM_LEAD_MIN
 #define MM_LEAD_MIN 8  // a group's wildcards from which a leading run is looked for
 #endif
@@ -577,6 +582,13 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
   __shared__ uint32_t sh_K, sh_types, sh_matched;
   // leading-run windows (global-workspace variants only): 2 rings of 64 per warp
   __shared__ uint16_t lead_ring[SMEM ? 1 : NT / 32][128];
+  // data-parallel leading runs (global-workspace variants): the groups with
+  // a run, and per batch of four their representative, key, first exact
+  // receive, run length, message count and first wildcard after the run
+  __shared__ uint16_t sh_lead_list[SMEM ? 1 : kLeadList];
+  __shared__ uint32_t sh_nlead, sh_lg[4], sh_lfe[4], sh_lrl[4], sh_lmc[4], sh_lafter[4];
+  __shared__ uint32_t sh_lwarp[SMEM ? 1 : NT / 32][4];
+  __shared__ uint64_t sh_lgk[4];
   constexpr int NW = NT / 32;
   // each side of the queue is cut in QP parts, placed by one warp each in P6
   // (4 for 256 threads; 16 for the 1024-thread deep-endpoint CTAs)
@@ -969,6 +981,136 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           ws.gwc[g] = 0;  // served
         }
         __syncthreads();
+#if MM_DP_LEAD
+        MM_PHASE(10);
+        if (lead_ok && L.lead_runw >= 0) {
+          // Leading runs, data-parallel: the r-th wildcard
+          // of group g's run (its wildcards posted before the first exact
+          // receive fe_g of any of its tuples) takes the group's r-th message
+          // in arrival order, for r < n_g = min(run length, group messages);
+          // the later run wildcards take nothing.  Up to four groups at a
+          // time, each rank a 16-bit field of one CTA-wide 64-bit scan: one
+          // scan over the wildcards (run ranks), one over the messages
+          // (group ranks), and every pair resolved in parallel -- no chain.
+          // The claims on tuple k are then its first m_k list entries, so
+          // message j = list_k[c] logs its wildcard at wlog[start_k + c].
+          uint16_t* runw = reinterpret_cast<uint16_t*>(base + L.lead_runw);
+          if (tid == 0) sh_nlead = 0;
+          __syncthreads();
+          for (uint32_t k = tid; k < K; k += NT)
+            if (ws.gwc[k] >= MM_LEAD_MIN) sh_lead_list[atomicAdd(&sh_nlead, 1u) & (kLeadList - 1)] = (uint16_t)k;
+          __syncthreads();
+          const uint32_t nlead = sh_nlead;
+          for (uint32_t b0 = 0; b0 < nlead && nlead <= kLeadList; b0 += 4) {
+            const uint32_t nb = min(4u, nlead - b0);
+            if ((uint32_t)tid < nb) {
+              const uint32_t g = sh_lead_list[b0 + tid];
+              sh_lg[tid] = g;
+              sh_lgk[tid] = ws.keyhdr[g] & gmsk;
+              sh_lfe[tid] = 0xFFFFFFFFu;
+              sh_lafter[tid] = W;
+            }
+            __syncthreads();
+            // first exact receive of each group: every tuple tests its group key
+            for (uint32_t k = tid; k < K; k += NT) {
+              const uint64_t gk = ws.keyhdr[k] & gmsk;
+              for (uint32_t t = 0; t < nb; t++)
+                if (gk == sh_lgk[t] && ws.key_rcnt[k]) atomicMin(&sh_lfe[t], (uint32_t)ws.rby_key[ws.key_rstart[k]]);
+            }
+            __syncthreads();
+            MM_PHASE(12);
+            // Ranks in (warp chunk, position) order: warp v owns a contiguous
+            // chunk, its lanes read consecutive elements (coalesced); pass 1
+            // counts each group's members per warp, the warps' exclusive
+            // prefixes come from shared totals, pass 2 ranks by ballot.
+            auto ranks = [&](uint32_t n, auto member, auto visit, uint32_t* totals) {
+              const uint32_t per = (n + NW - 1) / NW, c0 = min(n, warp * per), c1 = min(n, c0 + per);
+              uint32_t cnt[4] = {0, 0, 0, 0};
+              for (uint32_t y = c0; y < c1; y += 32) {
+                const uint32_t t = y + lane < c1 ? member(y + lane) : 4u;
+#pragma unroll
+                for (int q = 0; q < 4; q++) cnt[q] += __popc(__ballot_sync(kFull, t == (uint32_t)q));
+              }
+              if (lane < 4) sh_lwarp[warp][lane] = cnt[lane];
+              __syncthreads();
+              uint32_t run[4];
+#pragma unroll
+              for (int q = 0; q < 4; q++) {
+                run[q] = 0;
+                for (int v = 0; v < warp; v++) run[q] += sh_lwarp[v][q];
+              }
+              if (tid < 4) {
+                uint32_t all = 0;
+                for (int v = 0; v < NW; v++) all += sh_lwarp[v][tid];
+                totals[tid] = all;
+              }
+              for (uint32_t y = c0; y < c1; y += 32) {
+                const uint32_t yy = y + lane;
+                const uint32_t t = yy < c1 ? member(yy) : 4u;
+                uint32_t mine = 0;
+#pragma unroll
+                for (int q = 0; q < 4; q++) {
+                  const uint32_t bq = __ballot_sync(kFull, t == (uint32_t)q);
+                  if (t == (uint32_t)q) mine = run[q] + __popc(bq & lt);
+                  run[q] += __popc(bq);
+                }
+                if (t < 4u) visit(yy, t, mine);  // one visit per lane and step, whatever its group
+              }
+              __syncthreads();
+            };
+            // run ranks of the wildcards
+            ranks(
+                W,
+                [&](uint32_t x) -> uint32_t {
+                  const uint32_t g = ws.w_grp[x];
+                  for (uint32_t t = 0; t < nb; t++)
+                    if (g == sh_lg[t]) {
+                      if (ws.wl[x] < sh_lfe[t]) return t;
+                      atomicMin(&sh_lafter[t], x);
+                    }
+                  return 4u;
+                },
+                [&](uint32_t x, uint32_t t, uint32_t r) { runw[t * (uint32_t)a.R.cap + r] = (uint16_t)x; }, sh_lrl);
+            MM_PHASE(15);
+            // group ranks of the messages; pairs resolved at once
+            ranks(
+                nm,
+                [&](uint32_t j) -> uint32_t {
+                  const uint64_t mh = MS.hdr(j) & gmsk;
+                  for (uint32_t t = 0; t < nb; t++)
+                    if (mh == sh_lgk[t]) return t;
+                  return 4u;
+                },
+                [&](uint32_t j, uint32_t t, uint32_t r) {
+                  if (r < sh_lrl[t]) {
+                    const uint32_t x = runw[t * (uint32_t)a.R.cap + r];
+                    const uint32_t k = ws.msg_key[j], st = ws.key_start[k];
+                    uint32_t lo = 0, hi = ws.key_cnt[k];  // j's place in list_k
+                    while (lo < hi) {
+                      const uint32_t mid = (lo + hi) >> 1;
+                      if (ws.by_key[st + mid] < j) lo = mid + 1;
+                      else hi = mid;
+                    }
+                    ws.recv_res[x] = (uint16_t)j;
+                    ws.wlog[st + lo] = ws.wl[x];
+                    inc16(&ws.key_c[k]);
+                  }
+                },
+                sh_lmc);
+            // run wildcards beyond the group's messages take nothing; the
+            // chain continues after the run
+            for (uint32_t t = 0; t < nb; t++)
+              for (uint32_t r = sh_lmc[t] + tid; r < sh_lrl[t]; r += NT) ws.recv_res[runw[t * (uint32_t)a.R.cap + r]] = kNone;
+            if ((uint32_t)tid < nb) {
+              const uint32_t g = sh_lg[tid];
+              ws.gwc[g] -= sh_lrl[tid];
+              ws.gfirst[g] = sh_lafter[tid];
+            }
+            __syncthreads();
+            MM_PHASE(3);
+          }
+        }
+#endif
         MM_PHASE(10);
         // warp v serves the groups g % NW == v that still have wildcards (the
         // representatives are enumerated directly: no scan of the wildcards)
@@ -1007,7 +1149,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             uint32_t left = ws.gwc[gg];
             uint32_t x0 = ws.gfirst[gg];
             if (kn <= 32) {
-              if (lead_ok && left >= MM_LEAD_MIN) {
+              if (lead_ok && !MM_DP_LEAD && left >= MM_LEAD_MIN) {
                 // first exact receive of any of the group's tuples
                 uint32_t fe = 0xFFFFFFFFu;
                 if (lane < (int)kn && ws.key_rcnt[mine]) fe = ws.rby_key[ws.key_rstart[mine]];
@@ -1209,6 +1351,9 @@ FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
   // global workspace: wlog in a region of its own, so that msg_key stays
   // alive in P7 for the groups' leading runs (lead_run)
   if (!L.in_smem) L.wlog = take(2 * mcap);
+  // global workspace: the run positions of the data-parallel leading runs
+  // (4 groups at a time, up to rcap wildcards each)
+  L.lead_runw = L.in_smem ? -1 : take(8 * rcap);
   L.total = off;
   if (!L.in_smem) {
     const int64_t sb = r16(2 * mcap), sr = r16(2 * rcap);

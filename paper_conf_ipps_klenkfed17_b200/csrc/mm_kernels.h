@@ -38,6 +38,7 @@ struct FifoLayout {
   // rby_key, wl, recv_key) staged in the CTA's shared memory when they fit
   int64_t stage_bytes = 0, st_by_key = 0, st_rby_key = 0, st_wl = 0, st_recv_key = 0;
   int64_t st_wlog = -1;  // staged wildcard-claim log (P7..P8) when it fits, else -1
+  int64_t lead_runw = -1;  // global workspace: run positions of the data-parallel leading runs, else -1
 };
 FifoLayout fifo_layout(int64_t rcap, int64_t mcap);
 int fifo_grid(const FifoLayout& L, int n_ep);

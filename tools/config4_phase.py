@@ -20,9 +20,11 @@ for it in range(3):
     eng.reset(); eng.post_recvs(rh, None, ro); eng.push_msgs(mh, None, mo); eng.match_batch(orc, omc)
     torch.cuda.synchronize()
     L.mm_debug_phase_cycles(buf.ctypes.data, 1)
-names = ["prologue", "P1 stage", "P2 insert", "P3 ids", "P4 classify", "P5 scans", "P6 place", "P7 wildcards",
-         "P8 resolve+out", "P9 msg compact", "P7a group setup", "P7 K<=32 chain"]
-tot = buf[:12].sum()
+names = ["prologue", "P1 stage", "P2 insert", "P7 lead: messages", "P4 classify", "P5 scans", "P6 place",
+         "P7 wildcards", "P8 resolve+out", "P9 msg compact", "P7a group setup", "P7 K<=32 chain", "P7 lead: fe",
+         "-", "-", "P7 lead: run ranks"]
+tot = buf[:13].sum() + buf[15]
 for i, nm in enumerate(names):
-    print("%-16s %9.0f cycles  %5.1f%%" % (nm, buf[i], 100.0 * buf[i] / max(tot, 1)))
+    if nm != "-":
+        print("%-20s %9.0f cycles  %5.1f%%" % (nm, buf[i], 100.0 * buf[i] / max(tot, 1)))
 print("total %.0f cycles (one endpoint), K<=32 chain %d, group path %d" % (tot, buf[13], buf[14]))
