@@ -32,10 +32,26 @@
 //     per 4*NT receives);
 //  P9 unmatched messages compacted in arrival order (same).
 // Exact by construction: no ties (arrival indices are unique).
+#include <cooperative_groups.h>
+
 #include "mm_kernels.h"
 #include "mm_smem.cuh"
 
 namespace mm {
+namespace cg = cooperative_groups;
+
+#ifndef MM_DEEP_THREADS
+#define MM_DEEP_THREADS 1024  // threads per deep-queue endpoint CTA
+#endif
+#ifndef MM_DEEP_CS
+#define MM_DEEP_CS 8  // CTAs per deep endpoint's cluster (1: one CTA; A/B on configs[4]: 2 0.148, 4 0.110, 8 0.100, 16 0.124 ms)
+#endif
+#ifndef MM_CLUSTER_QP
+#define MM_CLUSTER_QP 32  // parts per side placed in P6 by a cluster (A/B: 16 0.108, 32 0.100, 64 0.101 ms on configs[4])
+#endif
+#ifndef MM_CLUSTER_STAGE
+#define MM_CLUSTER_STAGE 0  // 1: a cluster's hottest arrays staged in CTA 0's shared memory (A/B: 0.144 vs 0.100 ms in L2)
+#endif
 
 // Optional per-phase cycle accounting (build with -DMM_PHASE_TIMING; read by
 // mm_debug_phase_cycles).  Thread 0 of each CTA adds clock64 deltas.
@@ -44,7 +60,7 @@ __device__ unsigned long long g_phase_cycles[16];
 __device__ unsigned int g_ep_dbg[16384 * 4];  // per endpoint: P7 cycles, K, W, groups served
 #define MM_PHASE(n)                                                      \
   do {                                                                  \
-    if (threadIdx.x == 0) {                                             \
+    if (vt == 0) {                                                      \
       const long long _t = clock64();                                   \
       atomicAdd(&g_phase_cycles[n], (unsigned long long)(_t - t_phase)); \
       t_phase = _t;                                                     \
@@ -575,27 +591,75 @@ constexpr uint32_t kLeadList = 1024;  // groups with a leading run handled per e
 #endif
 constexpr uint32_t kGroupMinK = MM_GROUP_MIN_K;
 
-template <int NT, bool SMEM>
+// Per-endpoint scalars of k_mpi_fifo; with CS > 1 only CTA 0's copy is used
+// (distributed shared memory).
+template <int LL, int CS>
+struct FifoShared {
+  uint32_t K, types, matched, nlead;
+  uint32_t lg[4], lfe[4], lrl[4], lmc[4], lafter[4];
+  uint64_t lgk[4];
+  uint64_t ctot[2][CS];  // CTA totals of the cluster scans
+  uint16_t lead_list[LL];
+};
+
+// The endpoint's barrier: the CTA's, or the cluster's (which also orders
+// shared, distributed-shared and global memory across the cluster).
+template <int CS>
+__device__ __forceinline__ void bar() {
+  if constexpr (CS > 1) cg::this_cluster().sync();
+  else __syncthreads();
+}
+// Publication fence before a tuple's id becomes visible (P2, group table).
+template <int CS>
+__device__ __forceinline__ void fence() {
+  if constexpr (CS > 1) __threadfence();
+  else __threadfence_block();
+}
+// Exclusive scan over all threads of the endpoint (CTA, or cluster in rank
+// order): the CTA scan, then the CTA totals through CTA 0's shared memory.
+template <int NT, int CS>
+__device__ __forceinline__ uint64_t cscan64(uint64_t v, uint64_t* sm, uint64_t* ctot, int crank, uint64_t* total) {
+  uint64_t loc;
+  const uint64_t ex = scan64<NT>(v, sm, &loc);
+  if constexpr (CS == 1) {
+    (void)ctot;
+    (void)crank;
+    *total = loc;
+    return ex;
+  } else {
+    if (threadIdx.x == 0) ctot[crank] = loc;
+    cg::this_cluster().sync();
+    uint64_t pre = 0, tot = 0;
+#pragma unroll
+    for (int c = 0; c < CS; c++) {
+      const uint64_t x = ctot[c];
+      pre += c < crank ? x : 0ull;
+      tot += x;
+    }
+    *total = tot;
+    return pre + ex;
+  }
+}
+
+template <int NT, bool SMEM, int CS>
 __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_t* gws) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   __shared__ uint64_t scan_sm[2][NT / 32];
-  __shared__ uint32_t sh_K, sh_types, sh_matched;
+
   // leading-run windows (global-workspace variants only): 2 rings of 64 per warp
   __shared__ uint16_t lead_ring[SMEM ? 1 : NT / 32][128];
-  // data-parallel leading runs (global-workspace variants): the groups with
-  // a run, and per batch of four their representative, key, first exact
-  // receive, run length, message count and first wildcard after the run
-  __shared__ uint16_t sh_lead_list[SMEM ? 1 : kLeadList];
-  __shared__ uint32_t sh_nlead, sh_lg[4], sh_lfe[4], sh_lrl[4], sh_lmc[4], sh_lafter[4];
-  __shared__ uint32_t sh_lwarp[SMEM ? 1 : NT / 32][4];
-  __shared__ uint64_t sh_lgk[4];
-  constexpr int NW = NT / 32;
+  // the endpoint's scalars, incl. the data-parallel leading runs' groups
+  // (CS > 1: CTA 0's copy, reached through distributed shared memory)
+  __shared__ FifoShared<SMEM ? 1 : kLeadList, CS> shl;
+  constexpr int VT = NT * CS;
+  constexpr int VW = VT / 32;
   // each side of the queue is cut in QP parts, placed by one warp each in P6
-  // (4 for 256 threads; 16 for the 1024-thread deep-endpoint CTAs)
-  constexpr int QP = NT / 64;
-  static_assert(QP >= 4 && 2 * QP <= NW, "two sides of QP parts, one warp per part");
+  // (4 for 256 threads; 16 for the 1024-thread deep-endpoint CTAs; 16 CS for
+  // a cluster)
+  constexpr int QP = CS > 1 ? MM_CLUSTER_QP : VT / 64;
+  static_assert(QP >= 4 && 2 * QP <= VW, "two sides of QP parts, one warp per part");
   // compile-time choice, so that shared-memory accesses compile to LDS/STS/ATOMS
-  uint8_t* base = SMEM ? smem_raw : gws + (size_t)blockIdx.x * L.total;
+  uint8_t* base = SMEM ? smem_raw : gws + (size_t)(CS > 1 ? blockIdx.x / CS : blockIdx.x) * L.total;
   FifoWs ws = carve(base, L);
   if (!SMEM && L.stage_bytes > 0) {  // deep queues: the hottest arrays in shared memory
     ws.by_key = reinterpret_cast<uint16_t*>(smem_raw + L.st_by_key);
@@ -603,15 +667,35 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     ws.wl = reinterpret_cast<uint16_t*>(smem_raw + L.st_wl);
     ws.recv_key = reinterpret_cast<uint16_t*>(smem_raw + L.st_recv_key);
     if (L.st_wlog >= 0) ws.wlog = reinterpret_cast<uint16_t*>(smem_raw + L.st_wlog);
+    if constexpr (CS > 1) {  // the cluster's staged arrays: CTA 0's, through DSMEM
+      auto cl = cg::this_cluster();
+      ws.by_key = cl.map_shared_rank(ws.by_key, 0);
+      ws.rby_key = cl.map_shared_rank(ws.rby_key, 0);
+      ws.wl = cl.map_shared_rank(ws.wl, 0);
+      ws.recv_key = cl.map_shared_rank(ws.recv_key, 0);
+      if (L.st_wlog >= 0) ws.wlog = cl.map_shared_rank(ws.wlog, 0);
+    }
   }
+  // CS > 1: one endpoint per thread-block cluster of CS CTAs (deep queues):
+  // the CTAs' threads form one virtual CTA of VT threads (vt, vw), data-
+  // parallel loops and parts are spread over all of them, barriers are
+  // cluster barriers, scans add the CTAs' totals through distributed shared
+  // memory, and the per-endpoint scalars live in CTA 0's shared memory.
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int crank = CS > 1 ? (int)cg::this_cluster().block_rank() : 0;
+  const int vt = crank * NT + tid, vw = vt >> 5;
+  const int cid = CS > 1 ? (int)(blockIdx.x / CS) : (int)blockIdx.x;
+  const int ncl = CS > 1 ? (int)(gridDim.x / CS) : (int)gridDim.x;
+  FifoShared<SMEM ? 1 : kLeadList, CS>* Sp = &shl;
+  if constexpr (CS > 1) Sp = cg::this_cluster().map_shared_rank(&shl, 0);
+  auto& S = *Sp;
   const uint32_t lt = lanemask_lt();
   const uint32_t H = L.H, hmask = L.H - 1;
 
 #ifdef MM_PHASE_TIMING
   long long t_phase = clock64();
 #endif
-  for (int e = a.ep0 + blockIdx.x; e < a.n_ep; e += gridDim.x) {
+  for (int e = a.ep0 + cid; e < a.n_ep; e += ncl) {
     const int64_t rres = a.R.q_len[e], mres = a.M.q_len[e];
     const int64_t rpb = a.R.pend_begin(e), mpb = a.M.pend_begin(e);
     const int64_t nr64 = rres + a.R.pend_count(e), nm64 = mres + a.M.pend_count(e);
@@ -619,9 +703,9 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     if (nr64 > a.R.cap || nm64 > a.M.cap || obase + nr64 > a.out_cap) {
       // the endpoint's batch is rejected (mm.h): its receives are reported
       // unmatched when the output holds them, its queues are left as they were
-      if (tid == 0) atomicOr(a.err, kErrCapacity);
+      if (vt == 0) atomicOr(a.err, kErrCapacity);
       if (obase + nr64 <= a.out_cap)
-        for (int64_t i = tid; i < nr64; i += blockDim.x) {
+        for (int64_t i = vt; i < nr64; i += VT) {
           a.out_rc[obase + i] = a.R.cookie(e, i, rres, rpb);
           a.out_mc[obase + i] = (int64_t)MM_NO_MATCH;
         }
@@ -647,38 +731,38 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     uint64_t hv[4];
 #pragma unroll
     for (int u = 0; u < 4; u++) {
-      const uint32_t j = tid + u * NT;
+      const uint32_t j = vt + u * VT;
       hv[u] = j < nm ? MS.hdr(j) : 0ull;
     }
 
     // P1 -------------------------------------------------------------------
-    for (uint32_t s = tid; s < H / 4; s += NT) reinterpret_cast<uint4*>(ws.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
-    for (uint32_t k = tid; k < (nm + 31) / 32; k += NT) ws.matched[k] = 0u;
+    for (uint32_t s = vt; s < H / 4; s += VT) reinterpret_cast<uint4*>(ws.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
+    for (uint32_t k = vt; k < (nm + 31) / 32; k += VT) ws.matched[k] = 0u;
     if (SMEM) {  // per-quarter counts cleared in bulk (in HBM the CAS winners clear their rows)
       const uint32_t n16 = (uint32_t)(2 * QP * ws.mcap * 2 / 16);
-      for (uint32_t s = tid; s < n16; s += NT) reinterpret_cast<uint4*>(ws.pcnt)[s] = make_uint4(0u, 0u, 0u, 0u);
+      for (uint32_t s = vt; s < n16; s += VT) reinterpret_cast<uint4*>(ws.pcnt)[s] = make_uint4(0u, 0u, 0u, 0u);
     }
-    if (tid == 0) {
-      sh_matched = 0;
-      sh_K = 0;
-      sh_types = 0;
+    if (vt == 0) {
+      S.matched = 0;
+      S.K = 0;
+      S.types = 0;
     }
-    __syncthreads();
+    bar<CS>();
     MM_PHASE(1);
     // P2 -------------------------------------------------------------------
     // insert message tuples; the CAS winner of a slot takes the next dense
     // tuple id and initialises the tuple's entries before publishing it
-    for (uint32_t j0 = tid; j0 < nm; j0 += 4 * NT) {
-      if (j0 != (uint32_t)tid) {
+    for (uint32_t j0 = vt; j0 < nm; j0 += 4 * VT) {
+      if (j0 != (uint32_t)vt) {
 #pragma unroll
         for (int u = 0; u < 4; u++) {  // read once from HBM, four loads in flight
-          const uint32_t j = j0 + u * NT;
+          const uint32_t j = j0 + u * VT;
           hv[u] = j < nm ? MS.hdr(j) : 0ull;
         }
       }
 #pragma unroll
       for (int u = 0; u < 4; u++) {
-        const uint32_t j = j0 + u * NT;
+        const uint32_t j = j0 + u * VT;
         if (j >= nm) break;
         const uint64_t h = hv[u];
         uint32_t s, fp;
@@ -689,21 +773,24 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           if (o == kEmpty32) {
             o = atomicCAS(&ws.table[s], kEmpty32, (fp << 16) | kPending16);
             if (o == kEmpty32) {  // this message opens the tuple
-              id = atomicAdd(&sh_K, 1u);
+              id = atomicAdd(&S.K, 1u);
               ws.keyhdr[id] = h;
               if (!SMEM) {
 #pragma unroll
                 for (int q = 0; q < 2 * QP; q++) ws.pcnt[q * ws.mcap + id] = 0;
               }
               ws.key_c[id] = 0;
-              __threadfence_block();
+              fence<CS>();
               *reinterpret_cast<volatile uint32_t*>(&ws.table[s]) = (fp << 16) | id;
               break;
             }
           }
           if ((o >> 16) == fp) {
             while ((o & 0xFFFFu) == kPending16) o = *reinterpret_cast<volatile uint32_t*>(&ws.table[s]);
-            if (ws.keyhdr[o & 0xFFFFu] == h) {
+            // (a cluster's CTAs do not share an L1: the header just published
+            // by another SM is read from L2)
+            const uint64_t kh = CS > 1 ? __ldcg(&ws.keyhdr[o & 0xFFFFu]) : ws.keyhdr[o & 0xFFFFu];
+            if (kh == h) {
               id = o & 0xFFFFu;
               break;
             }
@@ -717,31 +804,31 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     // the first round of receive headers, requested before the barrier
 #pragma unroll
     for (int u = 0; u < 4; u++) {
-      const uint32_t i = tid + u * NT;
+      const uint32_t i = vt + u * VT;
       hv[u] = i < nr ? RS.hdr(i) : 0ull;
     }
-    __syncthreads();
+    bar<CS>();
     MM_PHASE(2);
-    const uint32_t K = sh_K;
+    const uint32_t K = S.K;
     // P4 -------------------------------------------------------------------
-    for (uint32_t i0 = tid; i0 < nr; i0 += 4 * NT) {
-      if (i0 != (uint32_t)tid) {
+    for (uint32_t i0 = vt; i0 < nr; i0 += 4 * VT) {
+      if (i0 != (uint32_t)vt) {
 #pragma unroll
         for (int u = 0; u < 4; u++) {  // four independent HBM loads in flight
-          const uint32_t i = i0 + u * NT;
+          const uint32_t i = i0 + u * VT;
           hv[u] = i < nr ? RS.hdr(i) : 0ull;
         }
       }
 #pragma unroll
       for (int u = 0; u < 4; u++) {
-        const uint32_t i = i0 + u * NT;
+        const uint32_t i = i0 + u * VT;
         if (i >= nr) break;
         const uint64_t h = hv[u];
         uint16_t rk;
         const bool anys = (uint32_t)h == MM_ANY_SOURCE, anyt = ((uint32_t)(h >> 32) & 0xFFFFu) == MM_ANY_TAG;
         if (anys || anyt) {
           rk = kWild;
-          atomicOr(&sh_types, 1u << ((anys ? 1u : 0u) | (anyt ? 2u : 0u)));
+          atomicOr(&S.types, 1u << ((anys ? 1u : 0u) | (anyt ? 2u : 0u)));
         } else {
           rk = kNone;
           uint32_t s, fp;
@@ -762,8 +849,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         ws.recv_key[i] = rk;
       }
     }
-    __syncthreads();
-    const uint32_t types = sh_types;
+    bar<CS>();
+    const uint32_t types = S.types;
     const bool grouped = __popc(types) == 1 && K > kGroupMinK;
     MM_PHASE(4);
     // P5 -------------------------------------------------------------------
@@ -771,8 +858,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     {
       // tuple list starts for messages (bits 0..15) and exact receives
       // (16..31), wildcard count (32..63), in one scan
-      const uint32_t per = (K + NT - 1) / NT;
-      const uint32_t k0 = min(K, tid * per), k1 = min(K, k0 + per);
+      const uint32_t per = (K + VT - 1) / VT;
+      const uint32_t k0 = min(K, vt * per), k1 = min(K, k0 + per);
       uint32_t c = 0;
       for (uint32_t k = k0; k < k1; k++) {
         // exclusive prefix over the parts: the base rank of each part
@@ -789,16 +876,16 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         ws.key_rcnt[k] = (uint16_t)rr;
         c += rm | (rr << 16);
       }
-      const uint32_t rper = (nr + NT - 1) / NT;
-      const uint32_t i0 = min(tid * rper, nr), i1 = min(i0 + rper, nr);
+      const uint32_t rper = (nr + VT - 1) / VT;
+      const uint32_t i0 = min(vt * rper, nr), i1 = min(i0 + rper, nr);
       uint32_t wc = 0;
       if (types)
         for (uint32_t i = i0; i < i1; i++) wc += ws.recv_key[i] == kWild;
       // the tuple table is free from here on: clear it for the group table
       if (grouped)
-        for (uint32_t s = tid; s < H / 4; s += NT) reinterpret_cast<uint4*>(ws.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
+        for (uint32_t s = vt; s < H / 4; s += VT) reinterpret_cast<uint4*>(ws.table)[s] = make_uint4(~0u, ~0u, ~0u, ~0u);
       uint64_t tot;
-      const uint64_t ex = scan64<NT>((uint64_t)c | ((uint64_t)wc << 32), scan_sm[0], &tot);
+      const uint64_t ex = cscan64<NT, CS>((uint64_t)c | ((uint64_t)wc << 32), scan_sm[0], S.ctot[0], crank, &tot);
       uint32_t st = (uint32_t)ex;
       for (uint32_t k = k0; k < k1; k++) {
         ws.key_start[k] = (uint16_t)st;
@@ -815,7 +902,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         }
       W = (uint32_t)(tot >> 32);
     }
-    __syncthreads();
+    bar<CS>();
     // header of the x-th wildcard (staged for the first wcap of them)
     auto hdrof = [&](uint32_t x) -> uint64_t {
       return x < L.wcap ? ws.whdr[x] : RS.hdr(ws.wl[x]);
@@ -824,12 +911,12 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     // P6 -------------------------------------------------------------------
     // warps 0..QP-1 place the QP parts of the messages, warps QP..2QP-1
     // those of the receives; each part starts from its base ranks
-    if (warp < 2 * QP) {
-      const bool msg_side = warp < QP;
-      const int q = warp % QP;
+    if (vw < 2 * QP) {
+      const bool msg_side = vw < QP;
+      const int q = vw % QP;
       const uint32_t n = msg_side ? nm : nr;
       const uint32_t x0 = (uint32_t)(((uint64_t)n * q + QP - 1) / QP), x1 = (uint32_t)(((uint64_t)n * (q + 1) + QP - 1) / QP);
-      uint16_t* running = ws.pcnt + (int64_t)warp * ws.mcap;
+      uint16_t* running = ws.pcnt + (int64_t)vw * ws.mcap;
       if (msg_side) {
         place_in_order(
             (int64_t)(x1 - x0), [&](int64_t x) { return (uint32_t)ws.msg_key[x0 + x]; }, ws.key_start, running,
@@ -844,16 +931,16 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             lane, lt, K);
       }
     }
-    __syncthreads();
+    bar<CS>();
     MM_PHASE(6);
 #ifdef MM_PHASE_TIMING
     const long long t_p7 = clock64();
     __shared__ unsigned int sh_groups;
-    if (tid == 0) sh_groups = 0;
+    if (vt == 0) sh_groups = 0;
 #endif
     // P7: wildcards -------------------------------------------------------
-    // sequential chains run on the highest warp ids: the issue arbiter serves
-    // higher warp ids first, so the critical path is not starved by the
+    // sequential chains run on the highest vw ids: the issue arbiter serves
+    // higher vw ids first, so the critical path is not starved by the
     // parallel phases of co-resident CTAs (B300_MICROARCH.md, arbiter)
     if (W > 0) {
       if (!grouped && K <= 32) {
@@ -862,32 +949,32 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         uint32_t* kmask = ws.gnext;
         uint16_t* kpre = reinterpret_cast<uint16_t*>(kmask + nch * 32);
         if ((int64_t)nch * 32 * 6 <= (int64_t)(L.recv_res - L.gnext)) {
-          for (uint32_t x = tid; x < nch * 32; x += NT) kmask[x] = 0u;
-          __syncthreads();
-          for (uint32_t i = tid; i < nr; i += NT) {
+          for (uint32_t x = vt; x < nch * 32; x += VT) kmask[x] = 0u;
+          bar<CS>();
+          for (uint32_t i = vt; i < nr; i += VT) {
             const uint32_t rk = ws.recv_key[i];
             if (rk < K) atomicOr(&kmask[(i >> 5) * 32 + rk], 1u << (i & 31u));
           }
-          __syncthreads();
-          if ((uint32_t)tid < K) {
+          bar<CS>();
+          if ((uint32_t)vt < K) {
             uint32_t run = 0;
             for (uint32_t ch = 0; ch < nch; ch++) {
-              kpre[ch * 32 + tid] = (uint16_t)run;
-              run += __popc(kmask[ch * 32 + tid]);
+              kpre[ch * 32 + vt] = (uint16_t)run;
+              run += __popc(kmask[ch * 32 + vt]);
             }
           }
-          __syncthreads();
-          if (warp == NW - 1) mask_chain(ws, kmask, kpre, K, W, hdrof, lane);
-        } else if (warp == NW - 1) {
+          bar<CS>();
+          if (vw == VW - 1) mask_chain(ws, kmask, kpre, K, W, hdrof, lane);
+        } else if (vw == VW - 1) {
           stream_chain(ws, ws.gnext, nr, K, W, hdrof, lane);  // gnext is free here
         }
         MM_PHASE(11);
 #ifdef MM_PHASE_TIMING
-        if (tid == 0) atomicAdd(&g_phase_cycles[13], 1ull);
+        if (vt == 0) atomicAdd(&g_phase_cycles[13], 1ull);
 #endif
       } else if (grouped) {
 #ifdef MM_PHASE_TIMING
-        if (tid == 0) atomicAdd(&g_phase_cycles[14], 1ull);
+        if (vt == 0) atomicAdd(&g_phase_cycles[14], 1ull);
 #endif
         // Wildcards of one type (all ANY_SOURCE, all ANY_TAG, or all both)
         // touch disjoint tuple groups {k : k & mask == r & mask}; groups are
@@ -900,7 +987,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         // group table: the first tuple of a group to win a slot represents it;
         // it initialises its group entries BEFORE publishing, so members that
         // find it may link themselves in at once (no pending state)
-        for (uint32_t k = tid; k < K; k += NT) {
+        for (uint32_t k = vt; k < K; k += VT) {
           ws.gwc[k] = 0;  // every tuple: nonzero after the wildcard pass = a representative with wildcards
           const uint64_t gk = ws.keyhdr[k] & gmsk;
           uint32_t s, fp;
@@ -911,7 +998,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
               ws.gnext[k] = kNone32;
               ws.gfirst[k] = kNone32;
               ws.gwc[k] = 0;
-              __threadfence_block();
+              fence<CS>();
               o = atomicCAS(&ws.table[s], kEmpty32, (fp << 16) | k);
               if (o == kEmpty32) break;  // k represents the group
             }
@@ -922,8 +1009,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             s = (s + 1) & hmask;
           }
         }
-        __syncthreads();
-        for (uint32_t x = tid; x < W; x += NT) {
+        bar<CS>();
+        for (uint32_t x = vt; x < W; x += VT) {
           const uint64_t rg = hdrof(x) & gmsk;
           uint32_t s, fp;
           slot_fp(rg, hmask, s, fp);
@@ -944,12 +1031,12 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             atomicAdd(&ws.gwc[g], 1u);
           }
         }
-        __syncthreads();
+        bar<CS>();
         // A group with ONE wildcard and few tuples needs no chain: its
         // wildcard takes the earliest head list_k[e_k(w)] over the group's
         // tuples (no earlier claims).  One thread per such group, all groups
         // at once; the warps below serve the rest.
-        for (uint32_t x = tid; x < W; x += NT) {
+        for (uint32_t x = vt; x < W; x += VT) {
           const uint32_t g = ws.w_grp[x];
           if (g == kNone || ws.gwc[g] != 1) continue;
           uint32_t kn = 0;
@@ -980,7 +1067,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           }
           ws.gwc[g] = 0;  // served
         }
-        __syncthreads();
+        bar<CS>();
 #if MM_DP_LEAD
         MM_PHASE(10);
         if (lead_ok && L.lead_runw >= 0) {
@@ -995,55 +1082,56 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           // The claims on tuple k are then its first m_k list entries, so
           // message j = list_k[c] logs its wildcard at wlog[start_k + c].
           uint16_t* runw = reinterpret_cast<uint16_t*>(base + L.lead_runw);
-          if (tid == 0) sh_nlead = 0;
-          __syncthreads();
-          for (uint32_t k = tid; k < K; k += NT)
-            if (ws.gwc[k] >= MM_LEAD_MIN) sh_lead_list[atomicAdd(&sh_nlead, 1u) & (kLeadList - 1)] = (uint16_t)k;
-          __syncthreads();
-          const uint32_t nlead = sh_nlead;
+          if (vt == 0) S.nlead = 0;
+          bar<CS>();
+          for (uint32_t k = vt; k < K; k += VT)
+            if (ws.gwc[k] >= MM_LEAD_MIN) S.lead_list[atomicAdd(&S.nlead, 1u) & (kLeadList - 1)] = (uint16_t)k;
+          bar<CS>();
+          const uint32_t nlead = S.nlead;
+          int lpar = 0;
           for (uint32_t b0 = 0; b0 < nlead && nlead <= kLeadList; b0 += 4) {
             const uint32_t nb = min(4u, nlead - b0);
-            if ((uint32_t)tid < nb) {
-              const uint32_t g = sh_lead_list[b0 + tid];
-              sh_lg[tid] = g;
-              sh_lgk[tid] = ws.keyhdr[g] & gmsk;
-              sh_lfe[tid] = 0xFFFFFFFFu;
-              sh_lafter[tid] = W;
+            if ((uint32_t)vt < nb) {
+              const uint32_t g = S.lead_list[b0 + vt];
+              S.lg[vt] = g;
+              S.lgk[vt] = ws.keyhdr[g] & gmsk;
+              S.lfe[vt] = 0xFFFFFFFFu;
+              S.lafter[vt] = W;
             }
-            __syncthreads();
+            bar<CS>();
             // first exact receive of each group: every tuple tests its group key
-            for (uint32_t k = tid; k < K; k += NT) {
+            for (uint32_t k = vt; k < K; k += VT) {
               const uint64_t gk = ws.keyhdr[k] & gmsk;
               for (uint32_t t = 0; t < nb; t++)
-                if (gk == sh_lgk[t] && ws.key_rcnt[k]) atomicMin(&sh_lfe[t], (uint32_t)ws.rby_key[ws.key_rstart[k]]);
+                if (gk == S.lgk[t] && ws.key_rcnt[k]) atomicMin(&S.lfe[t], (uint32_t)ws.rby_key[ws.key_rstart[k]]);
             }
-            __syncthreads();
+            bar<CS>();
             MM_PHASE(12);
-            // Ranks in (warp chunk, position) order: warp v owns a contiguous
+            // Ranks in (vw chunk, position) order: vw v owns a contiguous
             // chunk, its lanes read consecutive elements (coalesced); pass 1
-            // counts each group's members per warp, the warps' exclusive
+            // counts each group's members per vw, the warps' exclusive
             // prefixes come from shared totals, pass 2 ranks by ballot.
             auto ranks = [&](uint32_t n, auto member, auto visit, uint32_t* totals) {
-              const uint32_t per = (n + NW - 1) / NW, c0 = min(n, warp * per), c1 = min(n, c0 + per);
+              const uint32_t per = (n + VW - 1) / VW, c0 = min(n, vw * per), c1 = min(n, c0 + per);
               uint32_t cnt[4] = {0, 0, 0, 0};
               for (uint32_t y = c0; y < c1; y += 32) {
                 const uint32_t t = y + lane < c1 ? member(y + lane) : 4u;
 #pragma unroll
                 for (int q = 0; q < 4; q++) cnt[q] += __popc(__ballot_sync(kFull, t == (uint32_t)q));
               }
-              if (lane < 4) sh_lwarp[warp][lane] = cnt[lane];
-              __syncthreads();
+              // warps' counts as four 16-bit fields, one contribution per
+              // warp: the (cluster-wide) exclusive scan gives every warp the
+              // counts of the warps before it
+              const uint64_t mine4 = (uint64_t)cnt[0] | ((uint64_t)cnt[1] << 16) | ((uint64_t)cnt[2] << 32) |
+                                     ((uint64_t)cnt[3] << 48);
+              uint64_t tot4;
+              uint64_t ex4 = cscan64<NT, CS>(lane == 0 ? mine4 : 0ull, scan_sm[lpar], S.ctot[lpar], crank, &tot4);
+              lpar ^= 1;
+              ex4 = __shfl_sync(kFull, ex4, 0);
               uint32_t run[4];
 #pragma unroll
-              for (int q = 0; q < 4; q++) {
-                run[q] = 0;
-                for (int v = 0; v < warp; v++) run[q] += sh_lwarp[v][q];
-              }
-              if (tid < 4) {
-                uint32_t all = 0;
-                for (int v = 0; v < NW; v++) all += sh_lwarp[v][tid];
-                totals[tid] = all;
-              }
+              for (int q = 0; q < 4; q++) run[q] = (uint32_t)(ex4 >> (16 * q)) & 0xFFFFu;
+              if (vt < 4) totals[vt] = (uint32_t)(tot4 >> (16 * vt)) & 0xFFFFu;
               for (uint32_t y = c0; y < c1; y += 32) {
                 const uint32_t yy = y + lane;
                 const uint32_t t = yy < c1 ? member(yy) : 4u;
@@ -1056,7 +1144,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
                 }
                 if (t < 4u) visit(yy, t, mine);  // one visit per lane and step, whatever its group
               }
-              __syncthreads();
+              bar<CS>();
             };
             // run ranks of the wildcards
             ranks(
@@ -1064,13 +1152,13 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
                 [&](uint32_t x) -> uint32_t {
                   const uint32_t g = ws.w_grp[x];
                   for (uint32_t t = 0; t < nb; t++)
-                    if (g == sh_lg[t]) {
-                      if (ws.wl[x] < sh_lfe[t]) return t;
-                      atomicMin(&sh_lafter[t], x);
+                    if (g == S.lg[t]) {
+                      if (ws.wl[x] < S.lfe[t]) return t;
+                      atomicMin(&S.lafter[t], x);
                     }
                   return 4u;
                 },
-                [&](uint32_t x, uint32_t t, uint32_t r) { runw[t * (uint32_t)a.R.cap + r] = (uint16_t)x; }, sh_lrl);
+                [&](uint32_t x, uint32_t t, uint32_t r) { runw[t * (uint32_t)a.R.cap + r] = (uint16_t)x; }, S.lrl);
             MM_PHASE(15);
             // group ranks of the messages; pairs resolved at once
             ranks(
@@ -1078,11 +1166,11 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
                 [&](uint32_t j) -> uint32_t {
                   const uint64_t mh = MS.hdr(j) & gmsk;
                   for (uint32_t t = 0; t < nb; t++)
-                    if (mh == sh_lgk[t]) return t;
+                    if (mh == S.lgk[t]) return t;
                   return 4u;
                 },
                 [&](uint32_t j, uint32_t t, uint32_t r) {
-                  if (r < sh_lrl[t]) {
+                  if (r < S.lrl[t]) {
                     const uint32_t x = runw[t * (uint32_t)a.R.cap + r];
                     const uint32_t k = ws.msg_key[j], st = ws.key_start[k];
                     uint32_t lo = 0, hi = ws.key_cnt[k];  // j's place in list_k
@@ -1096,39 +1184,39 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
                     inc16(&ws.key_c[k]);
                   }
                 },
-                sh_lmc);
+                S.lmc);
             // run wildcards beyond the group's messages take nothing; the
             // chain continues after the run
             for (uint32_t t = 0; t < nb; t++)
-              for (uint32_t r = sh_lmc[t] + tid; r < sh_lrl[t]; r += NT) ws.recv_res[runw[t * (uint32_t)a.R.cap + r]] = kNone;
-            if ((uint32_t)tid < nb) {
-              const uint32_t g = sh_lg[tid];
-              ws.gwc[g] -= sh_lrl[tid];
-              ws.gfirst[g] = sh_lafter[tid];
+              for (uint32_t r = S.lmc[t] + vt; r < S.lrl[t]; r += VT) ws.recv_res[runw[t * (uint32_t)a.R.cap + r]] = kNone;
+            if ((uint32_t)vt < nb) {
+              const uint32_t g = S.lg[vt];
+              ws.gwc[g] -= S.lrl[vt];
+              ws.gfirst[g] = S.lafter[vt];
             }
-            __syncthreads();
+            bar<CS>();
             MM_PHASE(3);
           }
         }
 #endif
         MM_PHASE(10);
-        // warp v serves the groups g % NW == v that still have wildcards (the
+        // vw v serves the groups g % VW == v that still have wildcards (the
         // representatives are enumerated directly: no scan of the wildcards)
         // (on chip, MM_ENUM_ONCHIP=0: the warps scan the wildcards for group
         // leaders instead -- A/B switch)
-        const uint32_t v = (uint32_t)(NW - 1 - warp);
+        const uint32_t v = (uint32_t)(VW - 1 - vw);
         constexpr bool kEnum = !SMEM || MM_ENUM_ONCHIP;
         const uint32_t lim = kEnum ? K : W;
-        for (uint32_t b = kEnum ? v : 0u; b < lim; b += kEnum ? 32u * NW : 32u) {
+        for (uint32_t b = kEnum ? v : 0u; b < lim; b += kEnum ? 32u * VW : 32u) {
           uint32_t g;
           bool lead;
           if (kEnum) {
-            g = b + (uint32_t)lane * NW;
+            g = b + (uint32_t)lane * VW;
             lead = g < K && ws.gwc[g] != 0;
           } else {
             const uint32_t x = b + lane;
             g = x < W ? ws.w_grp[x] : kNone;
-            lead = g != kNone && g % NW == v && ws.gfirst[g] == x && ws.gwc[g] != 0;
+            lead = g != kNone && g % VW == v && ws.gfirst[g] == x && ws.gwc[g] != 0;
           }
           uint32_t leaders = __ballot_sync(kFull, lead);
           while (leaders) {
@@ -1170,7 +1258,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             }
           }
         }
-      } else if (warp == NW - 1) {
+      } else if (vw == VW - 1) {
         for (uint32_t x = 0; x < W; x++) {
           const uint32_t w = ws.wl[x];
           const uint64_t r = hdrof(x);
@@ -1178,9 +1266,9 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         }
       }
     }
-    __syncthreads();
+    bar<CS>();
 #ifdef MM_PHASE_TIMING
-    if (tid == 0 && e < 16384) {
+    if (vt == 0 && e < 16384) {
       g_ep_dbg[4 * e] = (unsigned int)(clock64() - t_p7);
       g_ep_dbg[4 * e + 1] = K;
       g_ep_dbg[4 * e + 2] = W;
@@ -1196,12 +1284,12 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       uint64_t* qrh = a.q_rh_w + (int64_t)e * a.R.cap;
       int64_t* qrc = a.q_rc_w + (int64_t)e * a.R.cap;
       uint32_t wr = 0, nmatch = 0;
-      for (uint32_t t0 = 0; t0 < nr; t0 += 4 * NT) {
+      for (uint32_t t0 = 0; t0 < nr; t0 += 4 * VT) {
         uint64_t fld = 0, rh[4];
         int64_t rcv[4];
 #pragma unroll
         for (int u = 0; u < 4; u++) {
-          const uint32_t i = t0 + u * NT + tid;
+          const uint32_t i = t0 + u * VT + vt;
           rh[u] = 0;
           rcv[u] = 0;
           if (i < nr) {
@@ -1240,7 +1328,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           }
         }
         uint64_t tot;
-        const uint64_t ex = scan64<NT>(fld, scan_sm[par], &tot);
+        const uint64_t ex = cscan64<NT, CS>(fld, scan_sm[par], S.ctot[par], crank, &tot);
         par ^= 1;
 #pragma unroll
         for (int u = 0; u < 4; u++)
@@ -1252,22 +1340,22 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         wr += fields_sum(tot);
       }
       for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
-      if (lane == 0 && nmatch) atomicAdd(&sh_matched, nmatch);
-      if (tid == 0) a.rres_w[e] = (int32_t)wr;
+      if (lane == 0 && nmatch) atomicAdd(&S.matched, nmatch);
+      if (vt == 0) a.rres_w[e] = (int32_t)wr;
     }
-    __syncthreads();  // matched bits complete
+    bar<CS>();  // matched bits complete
     MM_PHASE(8);
     // P9: compact the unexpected-message queue ------------------------------
     {
       uint64_t* qmh = a.q_mh_w + (int64_t)e * a.M.cap;
       int64_t* qmc = a.q_mc_w + (int64_t)e * a.M.cap;
       uint32_t wm = 0;
-      for (uint32_t t0 = 0; t0 < nm; t0 += 4 * NT) {
+      for (uint32_t t0 = 0; t0 < nm; t0 += 4 * VT) {
         uint64_t fld = 0, mh[4];
         int64_t mc[4];
 #pragma unroll
         for (int u = 0; u < 4; u++) {
-          const uint32_t j = t0 + u * NT + tid;
+          const uint32_t j = t0 + u * VT + vt;
           mh[u] = 0;
           mc[u] = 0;
           if (j < nm && !((ws.matched[j >> 5] >> (j & 31)) & 1u)) {
@@ -1277,7 +1365,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           }
         }
         uint64_t tot;
-        const uint64_t ex = scan64<NT>(fld, scan_sm[par], &tot);
+        const uint64_t ex = cscan64<NT, CS>(fld, scan_sm[par], S.ctot[par], crank, &tot);
         par ^= 1;
 #pragma unroll
         for (int u = 0; u < 4; u++)
@@ -1288,19 +1376,24 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           }
         wm += fields_sum(tot);
       }
-      if (tid == 0) {
+      if (vt == 0) {
         a.mres_w[e] = (int32_t)wm;
-        if (sh_matched) atomicAdd(a.n_matched, (unsigned long long)sh_matched);
+        if (S.matched) atomicAdd(a.n_matched, (unsigned long long)S.matched);
       }
     }
-    __syncthreads();  // the workspace is reused by the next endpoint
+    bar<CS>();  // the workspace is reused by the next endpoint
     MM_PHASE(9);
   }
 }
 
+#ifndef MM_DEEP_THREADS
+#define MM_DEEP_THREADS 1024  // threads per deep-queue endpoint CTA
+#endif
+
+constexpr int64_t kDeepClusterSMs = 144;  // clusters of MM_DEEP_CS SMs per launch, at most
 constexpr int64_t kFifoStageMax = 200 * 1024;  // shared memory for the staged arrays of deep endpoints
 
-FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
+FifoLayout fifo_layout(int64_t rcap, int64_t mcap, int n_ep) {
   FifoLayout L;
   int64_t H = 1;
   while (H < 2 * mcap) H <<= 1;
@@ -1340,7 +1433,11 @@ FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
   // workspace, 1024-thread deep-endpoint CTAs)
   const int64_t rows8 = grp > 16 * mcap ? grp : 16 * mcap;
   const bool fits = off + rows8 <= kFifoSmemMax;
-  const int64_t region = take(fits ? rows8 : (grp > 64 * mcap ? grp : 64 * mcap));
+  // global workspace: 16 parts per side (1024-thread CTA), or 16 per CTA of a
+  // cluster when every endpoint gets a cluster of its own (n_ep x CS <= SMs)
+  L.cluster = (!fits && MM_DEEP_CS > 1 && (int64_t)n_ep * MM_DEEP_CS <= kDeepClusterSMs) ? MM_DEEP_CS : 1;
+  const int64_t rowsg = 4 * (int64_t)(L.cluster > 1 ? MM_CLUSTER_QP : MM_DEEP_THREADS / 64) * mcap;
+  const int64_t region = take(fits ? rows8 : (grp > rowsg ? grp : rowsg));
   L.pcnt = region;
   L.gnext = region;
   L.gfirst = region + gn;
@@ -1375,7 +1472,7 @@ FifoLayout fifo_layout(int64_t rcap, int64_t mcap) {
 }
 
 int fifo_grid(const FifoLayout& L, int n_ep) {
-  if (L.in_smem) return n_ep;
+  if (L.in_smem || L.cluster > 1) return n_ep;  // CTAs / clusters (one workspace each)
   int g = 148 * 2;
   return n_ep < g ? n_ep : g;
 }
@@ -1396,33 +1493,64 @@ extern "C" int mm_debug_phase_cycles(unsigned long long* out, int reset) {
 }
 #endif
 
-#ifndef MM_DEEP_THREADS
-#define MM_DEEP_THREADS 1024  // threads per deep-queue endpoint CTA
-#endif
 cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws, cudaStream_t st) {
   if (a.n_ep <= a.ep0) return cudaSuccess;
   const int grid = fifo_grid(L, a.n_ep - a.ep0);
   cudaError_t err;
   if (L.in_smem) {
-    err = ensure_dyn_smem<k_mpi_fifo<256, true>>((size_t)L.total);
+    err = ensure_dyn_smem<k_mpi_fifo<256, true, 1>>((size_t)L.total);
     if (err != cudaSuccess) return err;
     count_launch();
-    k_mpi_fifo<256, true><<<grid, 256, (size_t)L.total, st>>>(a, L, nullptr);
+    k_mpi_fifo<256, true, 1><<<grid, 256, (size_t)L.total, st>>>(a, L, nullptr);
+  } else if (L.cluster > 1) {
+    FifoLayout LC = L;
+    if (!MM_CLUSTER_STAGE) LC.stage_bytes = 0;
+    // deep queues, few endpoints: one thread-block cluster of MM_DEEP_CS
+    // 1024-thread CTAs per endpoint (the data-parallel phases spread over
+    // MM_DEEP_CS SMs; the staged arrays in CTA 0's shared memory)
+    using KC = decltype(&k_mpi_fifo<MM_DEEP_THREADS, false, MM_DEEP_CS>);
+    KC kc = &k_mpi_fifo<MM_DEEP_THREADS, false, MM_DEEP_CS>;
+    if (LC.stage_bytes > 0) {
+      err = ensure_dyn_smem<k_mpi_fifo<MM_DEEP_THREADS, false, MM_DEEP_CS>>((size_t)LC.stage_bytes);
+      if (err != cudaSuccess) return err;
+    }
+#if MM_DEEP_CS > 8
+    static bool np_set = false;
+    if (!np_set) {
+      err = cudaFuncSetAttribute(kc, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+      if (err != cudaSuccess) return err;
+      np_set = true;
+    }
+#endif
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(grid * MM_DEEP_CS));
+    cfg.blockDim = dim3(MM_DEEP_THREADS);
+    cfg.dynamicSmemBytes = (size_t)LC.stage_bytes;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = MM_DEEP_CS;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    count_launch();
+    return cudaLaunchKernelEx(&cfg, kc, a, LC, gws);
   } else if (a.n_ep - a.ep0 <= 148) {
     // deep queues and at most one endpoint per SM: 1024 threads per endpoint
     // (the parallel phases over up to 24K elements shrink 4x; the chains
     // are unchanged)
     if (L.stage_bytes > 0) {
-      err = ensure_dyn_smem<k_mpi_fifo<MM_DEEP_THREADS, false>>((size_t)L.stage_bytes);
+      err = ensure_dyn_smem<k_mpi_fifo<MM_DEEP_THREADS, false, 1>>((size_t)L.stage_bytes);
       if (err != cudaSuccess) return err;
     }
     count_launch();
-    k_mpi_fifo<MM_DEEP_THREADS, false><<<grid, MM_DEEP_THREADS, (size_t)L.stage_bytes, st>>>(a, L, gws);
+    k_mpi_fifo<MM_DEEP_THREADS, false, 1><<<grid, MM_DEEP_THREADS, (size_t)L.stage_bytes, st>>>(a, L, gws);
   } else {
     FifoLayout L2 = L;  // several CTAs per SM: no staging
     L2.stage_bytes = 0;
     count_launch();
-    k_mpi_fifo<256, false><<<grid, 256, 0, st>>>(a, L2, gws);
+    k_mpi_fifo<256, false, 1><<<grid, 256, 0, st>>>(a, L2, gws);
   }
   return cudaGetLastError();
 }

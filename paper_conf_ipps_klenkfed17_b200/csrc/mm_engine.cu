@@ -369,7 +369,7 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
   if (ok && semantics == MM_SEM_MPI) {
     e->msg_slots = (e->mcap + 63) / 64 * 64;
     e->warp_words = (e->msg_slots + e->msg_slots / 64 + 3) / 4 * 4;  // headers + availability bits, 32 B aligned
-    e->fifo = fifo_layout(e->rcap, e->mcap);
+    e->fifo = fifo_layout(e->rcap, e->mcap, n_endpoints);
     if (!e->fifo.in_smem)
       ok = ensure(e->fifo_ws, (size_t)fifo_grid(e->fifo, n_endpoints) * (size_t)e->fifo.total) == cudaSuccess;
   }

@@ -39,8 +39,9 @@ struct FifoLayout {
   int64_t stage_bytes = 0, st_by_key = 0, st_rby_key = 0, st_wl = 0, st_recv_key = 0;
   int64_t st_wlog = -1;  // staged wildcard-claim log (P7..P8) when it fits, else -1
   int64_t lead_runw = -1;  // global workspace: run positions of the data-parallel leading runs, else -1
+  int cluster = 1;         // CTAs per deep endpoint (thread-block cluster), 1 = one CTA
 };
-FifoLayout fifo_layout(int64_t rcap, int64_t mcap);
+FifoLayout fifo_layout(int64_t rcap, int64_t mcap, int n_ep);
 int fifo_grid(const FifoLayout& L, int n_ep);
 cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws, cudaStream_t st);
 
