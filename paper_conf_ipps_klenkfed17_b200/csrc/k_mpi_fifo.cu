@@ -43,12 +43,16 @@ namespace cg = cooperative_groups;
 #ifndef MM_DEEP_THREADS
 #define MM_DEEP_THREADS 1024  // threads per deep-queue endpoint CTA
 #endif
+#ifndef MM_CLUSTER_THREADS
+#define MM_CLUSTER_THREADS 512  // threads per CTA of a deep endpoint's cluster (A/B, 8 CTAs: 1024 0.094, 512 0.085 ms; no spills)
+#endif
 #ifndef MM_DEEP_CS
-#define MM_DEEP_CS 8  // CTAs per deep endpoint's cluster (1: one CTA; A/B on configs[4]: 2 0.148, 4 0.110, 8 0.100, 16 0.124 ms)
+#define MM_DEEP_CS 8  // CTAs per deep endpoint's cluster (1: one CTA; A/B on configs[4], 1024-thread CTAs: 2 0.148, 4 0.110, 8 0.100, 16 0.124 ms)
 #endif
 #ifndef MM_CLUSTER_QP
 #define MM_CLUSTER_QP 32  // parts per side placed in P6 by a cluster (A/B: 16 0.108, 32 0.100, 64 0.101 ms on configs[4])
 #endif
+constexpr uint32_t kP6Smem = 2048;  // tuples whose P6 running counts a cluster keeps in shared memory
 #ifndef MM_CLUSTER_STAGE
 #define MM_CLUSTER_STAGE 0  // 1: a cluster's hottest arrays staged in CTA 0's shared memory (A/B: 0.144 vs 0.100 ms in L2)
 #endif
@@ -911,12 +915,26 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     // P6 -------------------------------------------------------------------
     // warps 0..QP-1 place the QP parts of the messages, warps QP..2QP-1
     // those of the receives; each part starts from its base ranks
-    if (vw < 2 * QP) {
-      const bool msg_side = vw < QP;
-      const int q = vw % QP;
+    // (a cluster spreads its 2 QP part-warps evenly over its CTAs)
+    constexpr int PS = VW / (2 * QP);
+    if (vw % PS == 0) {
+      const int pw = vw / PS;
+      const bool msg_side = pw < QP;
+      const int q = pw % QP;
       const uint32_t n = msg_side ? nm : nr;
       const uint32_t x0 = (uint32_t)(((uint64_t)n * q + QP - 1) / QP), x1 = (uint32_t)(((uint64_t)n * (q + 1) + QP - 1) / QP);
-      uint16_t* running = ws.pcnt + (int64_t)vw * ws.mcap;
+      uint16_t* running = ws.pcnt + (int64_t)pw * ws.mcap;
+      if constexpr (CS > 1) {
+        // a cluster's part-warps run their counts in the CTA's shared
+        // memory when the tuples fit (the rows start from the part's base
+        // ranks in L2)
+        if (K <= kP6Smem) {
+          uint16_t* row = reinterpret_cast<uint16_t*>(smem_raw) + (size_t)(warp / PS) * kP6Smem;
+          for (uint32_t k = lane; k < K; k += 32) row[k] = running[k];
+          __syncwarp();
+          running = row;
+        }
+      }
       if (msg_side) {
         place_in_order(
             (int64_t)(x1 - x0), [&](int64_t x) { return (uint32_t)ws.msg_key[x0 + x]; }, ws.key_start, running,
@@ -1386,9 +1404,6 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
   }
 }
 
-#ifndef MM_DEEP_THREADS
-#define MM_DEEP_THREADS 1024  // threads per deep-queue endpoint CTA
-#endif
 
 constexpr int64_t kDeepClusterSMs = 144;  // clusters of MM_DEEP_CS SMs per launch, at most
 constexpr int64_t kFifoStageMax = 200 * 1024;  // shared memory for the staged arrays of deep endpoints
@@ -1505,13 +1520,16 @@ cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws,
   } else if (L.cluster > 1) {
     FifoLayout LC = L;
     if (!MM_CLUSTER_STAGE) LC.stage_bytes = 0;
+    // P6's per-warp running counts: (2 QP / CS) part-warps per CTA
+    const int64_t p6 = (int64_t)(2 * MM_CLUSTER_QP / MM_DEEP_CS) * kP6Smem * 2;
+    const int64_t dyn = LC.stage_bytes > p6 ? LC.stage_bytes : p6;
     // deep queues, few endpoints: one thread-block cluster of MM_DEEP_CS
-    // 1024-thread CTAs per endpoint (the data-parallel phases spread over
+    // MM_CLUSTER_THREADS-thread CTAs per endpoint (the data-parallel phases spread over
     // MM_DEEP_CS SMs; the staged arrays in CTA 0's shared memory)
-    using KC = decltype(&k_mpi_fifo<MM_DEEP_THREADS, false, MM_DEEP_CS>);
-    KC kc = &k_mpi_fifo<MM_DEEP_THREADS, false, MM_DEEP_CS>;
-    if (LC.stage_bytes > 0) {
-      err = ensure_dyn_smem<k_mpi_fifo<MM_DEEP_THREADS, false, MM_DEEP_CS>>((size_t)LC.stage_bytes);
+    using KC = decltype(&k_mpi_fifo<MM_CLUSTER_THREADS, false, MM_DEEP_CS>);
+    KC kc = &k_mpi_fifo<MM_CLUSTER_THREADS, false, MM_DEEP_CS>;
+    {
+      err = ensure_dyn_smem<k_mpi_fifo<MM_CLUSTER_THREADS, false, MM_DEEP_CS>>((size_t)dyn);
       if (err != cudaSuccess) return err;
     }
 #if MM_DEEP_CS > 8
@@ -1524,8 +1542,8 @@ cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws,
 #endif
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)(grid * MM_DEEP_CS));
-    cfg.blockDim = dim3(MM_DEEP_THREADS);
-    cfg.dynamicSmemBytes = (size_t)LC.stage_bytes;
+    cfg.blockDim = dim3(MM_CLUSTER_THREADS);
+    cfg.dynamicSmemBytes = (size_t)dyn;
     cfg.stream = st;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeClusterDimension;
