@@ -267,6 +267,52 @@ def test_mpi_wide_headers_deep_endpoint(kind):
     assert_exact(g, o)
 
 
+@pytest.mark.parametrize("host,pipeline", [(False, None), (True, 2), ("in", 3)])
+@pytest.mark.parametrize("seed", [1, 2])
+def test_mpi_cluster_endpoints_multibatch(seed, host, pipeline):
+    """Deep endpoints on the thread-block-cluster variant (few endpoints,
+    queues too deep for one CTA's shared memory): ragged depths up to 3000,
+    both wildcard kinds, two communicators, unexpected messages, 3 batches
+    with residual queues; device buffers and the host-buffer pipeline (the
+    cluster kernel launched per endpoint range).  Bit-exact."""
+    rng = np.random.default_rng(seed)
+    q = synth.mpi_endpoints(seed + 40, n_ep=7, depth_r=3000, n_src=30, n_tag=9, p_any_src=0.08, p_any_tag=0.05,
+                            n_comm=2, ragged=True, p_unmatched=0.2)
+    batches = split_batches(q, 3, rng)
+    g, st = gpu_batches(MPI, 7, 3000, 3000, batches, host=host, pipeline=pipeline)
+    o, _ = oracle_batches(MPI, 7, batches)
+    assert_exact(g, o)
+    assert st["error"] == 0
+
+
+def test_mpi_cluster_capacity_overflow():
+    """Capacity overflow on the cluster variant: an endpoint over capacity is
+    flagged and reported unmatched; the others stay exact."""
+    q = synth.mpi_endpoints(77, n_ep=3, depth_r=2500, n_src=20, n_tag=5, ragged=False, p_unmatched=0.1)
+    big = synth.mpi_endpoints(78, n_ep=1, depth_r=2900, n_src=20, n_tag=5)
+    # endpoint 1 gets 2900 receives: over a 2600 capacity
+    eps = [q.endpoint(0), big.endpoint(0), q.endpoint(2)]
+    ro = np.cumsum([0] + [len(r) for r, _ in eps])
+    mo = np.cumsum([0] + [len(m) for _, m in eps])
+    rh = np.concatenate([r for r, _ in eps])
+    mh = np.concatenate([m[:2500] for _, m in eps])
+    mo = np.cumsum([0] + [min(len(m), 2500) for _, m in eps])
+    g, st = gpu_batches(MPI, 3, 2600, 2600, [(rh, None, ro, mh, None, mo)], out_cap=int(ro[-1]))
+    assert st["error"] != 0 and st["rc"] == 3
+    grc, gmc, _ = g[0]
+    assert np.all(gmc[ro[1]:ro[2]] == -1)
+    for e in (0, 2):
+        sub = synth.Queues(eps[e][0], [0, len(eps[e][0])], eps[e][1][:2500], [0, min(len(eps[e][1]), 2500)])
+        o, _ = oracle_batches(MPI, 1, single_batch(sub))
+        assert np.array_equal(gmc[ro[e]:ro[e + 1]], remap(o[0][1], mo[e]))
+
+
+def remap(omc, base):
+    """Oracle message cookies of a single-endpoint run -> the multi-endpoint
+    engine's (the engine numbers messages over all endpoints)."""
+    return np.where(omc >= 0, omc + base, omc)
+
+
 @pytest.mark.parametrize("case", ["worst", "mixed"])
 def test_mpi_maximum_capacity(case):
     """Queues at the MPI level's maximum capacity (MM_MPI_MAX_MSGS, global
