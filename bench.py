@@ -64,7 +64,7 @@ REGION_KERNELS = {
     "ordered": "k_part_hist + k_scan_* + k_part_scatter (both sides, 2 passes) + k_bucket_bounds + k_bucket_pair",
     "unordered": "k_part_hist + k_scan_* + k_part_scatter (both sides, 2 passes) + k_bucket_bounds + k_bucket_pop",
     "unordered_256m": "k_part_hist + k_scan_* + k_part_scatter (both sides) + k_bucket_bounds + k_bucket_pop",
-    "mpi_worst": "k_mpi_fifo (1024-thread deep-endpoint instantiation, one CTA)",
+    "mpi_worst": "k_mpi_fifo (deep-endpoint instantiation: one cluster of 8 512-thread CTAs)",
 }
 # PAPER.md's own rates (GTX1080 unless stated; other hardware: context, not target)
 PAPER_CONTEXT = {
@@ -343,8 +343,10 @@ def bench_mpi_worst(args, world, rank, peak):
     matches = int(cnt[1].item())
     # ncu counters of the 1024-thread deep-endpoint launch are keyed apart from
     # the configs[1] launch (same kernel name, different instantiation and work)
-    res.update(matches_per_step=matches, algo_bytes=8 * 2 * n + 16 * n, n_recv=n, n_msg=n, kernel="k_mpi_fifo",
-               capture="k_mpi_fifo_deep", sms_used=1, flush_ms=flush_ms)
+    # the endpoint runs on one thread-block cluster of 8 CTAs, one per SM
+    # (k_mpi_fifo.cu MM_DEEP_CS): the issue peak is that of 8 SMs
+    res.update(matches_per_step=matches, algo_bytes=8 * 2 * n + 16 * n, n_recv=n, n_msg=n,
+               kernel="k_mpi_fifo (8-CTA cluster)", capture="k_mpi_fifo_deep", sms_used=8, flush_ms=flush_ms)
     eng.close()
     out = finish_level(res, world, peak, "mpi_worst")
     out["_kernel_only"] = True

@@ -90,7 +90,9 @@ PartPlan part_plan(int64_t n_side) {
   int rest = pl.nb;
   int bits[kMaxPasses];
   int np = 0;
-  const int first = rest <= 8 ? rest : (rest <= 18 ? rest - rest / 2 : 8);  // <= 9: 2 x 512 keys
+  // two passes up to nb = 19 (9 + 10 bits: 2 x 512 keys, then 1024 keys per
+  // tile), three beyond
+  const int first = rest <= 8 ? rest : (rest <= 18 ? rest - rest / 2 : (rest == 19 ? 9 : 8));  // <= 9: 2 x 512 keys
   bits[np++] = first;
   rest -= first;
   const int later = (rest + 9) / 10;  // fewest later passes of <= 10 bits, bits spread evenly
