@@ -1517,21 +1517,21 @@ cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws,
     if (err != cudaSuccess) return err;
     count_launch();
     k_mpi_fifo<256, true, 1><<<grid, 256, (size_t)L.total, st>>>(a, L, nullptr);
-  } else if (L.cluster > 1) {
+    return cudaGetLastError();
+  }
+  if (L.cluster > 1) {
+    // deep queues, few endpoints: one thread-block cluster of MM_DEEP_CS
+    // MM_CLUSTER_THREADS-thread CTAs per endpoint (the data-parallel phases
+    // spread over MM_DEEP_CS SMs; the workspace in L2)
+    using KC = decltype(&k_mpi_fifo<MM_CLUSTER_THREADS, false, MM_DEEP_CS>);
+    KC kc = &k_mpi_fifo<MM_CLUSTER_THREADS, false, MM_DEEP_CS>;
     FifoLayout LC = L;
     if (!MM_CLUSTER_STAGE) LC.stage_bytes = 0;
     // P6's per-warp running counts: (2 QP / CS) part-warps per CTA
     const int64_t p6 = (int64_t)(2 * MM_CLUSTER_QP / MM_DEEP_CS) * kP6Smem * 2;
     const int64_t dyn = LC.stage_bytes > p6 ? LC.stage_bytes : p6;
-    // deep queues, few endpoints: one thread-block cluster of MM_DEEP_CS
-    // MM_CLUSTER_THREADS-thread CTAs per endpoint (the data-parallel phases spread over
-    // MM_DEEP_CS SMs; the staged arrays in CTA 0's shared memory)
-    using KC = decltype(&k_mpi_fifo<MM_CLUSTER_THREADS, false, MM_DEEP_CS>);
-    KC kc = &k_mpi_fifo<MM_CLUSTER_THREADS, false, MM_DEEP_CS>;
-    {
-      err = ensure_dyn_smem<k_mpi_fifo<MM_CLUSTER_THREADS, false, MM_DEEP_CS>>((size_t)dyn);
-      if (err != cudaSuccess) return err;
-    }
+    err = ensure_dyn_smem<k_mpi_fifo<MM_CLUSTER_THREADS, false, MM_DEEP_CS>>((size_t)dyn);
+    if (err != cudaSuccess) return err;
 #if MM_DEEP_CS > 8
     static bool np_set = false;
     if (!np_set) {
@@ -1553,8 +1553,11 @@ cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws,
     cfg.attrs = at;
     cfg.numAttrs = 1;
     count_launch();
-    return cudaLaunchKernelEx(&cfg, kc, a, LC, gws);
-  } else if (a.n_ep - a.ep0 <= 148) {
+    err = cudaLaunchKernelEx(&cfg, kc, a, LC, gws);
+    if (err == cudaSuccess) return cudaSuccess;
+    cudaGetLastError();  // no cluster of this shape can be scheduled: one CTA per endpoint instead
+  }
+  if (a.n_ep - a.ep0 <= 148) {
     // deep queues and at most one endpoint per SM: 1024 threads per endpoint
     // (the parallel phases over up to 24K elements shrink 4x; the chains
     // are unchanged)
