@@ -46,6 +46,14 @@ namespace cg = cooperative_groups;
 #ifndef MM_CLUSTER_THREADS
 #define MM_CLUSTER_THREADS 512  // threads per CTA of a deep endpoint's cluster (A/B, 8 CTAs: 1024 0.094, 512 0.085 ms; no spills)
 #endif
+#ifndef MM_P8_EARLY
+#define MM_P8_EARLY 0  // 1: P7's idle warps resolve the receives no chain can change (A/B on configs[1]: 15.8 vs 17.1 G/s -- they take issue slots from the chains)
+#endif
+constexpr uint16_t kEarlyHit = 0x8000u;   // recv_key: resolved early, matched message in the low 15 bits
+constexpr uint16_t kEarlyNone = 0xFFFDu;  // recv_key: resolved early, no match
+#ifndef MM_ONCHIP_PERSIST
+#define MM_ONCHIP_PERSIST 0  // on-chip variant: 0 = one CTA per endpoint, k = k x the resident CTA slots (A/B: 1 16.1, 2 16.2 vs 17.1 G/s)
+#endif
 #ifndef MM_DEEP_CS
 #define MM_DEEP_CS 8  // CTAs per deep endpoint's cluster (1: one CTA; A/B on configs[4], 1024-thread CTAs: 2 0.148, 4 0.110, 8 0.100, 16 0.124 ms)
 #endif
@@ -599,7 +607,7 @@ constexpr uint32_t kGroupMinK = MM_GROUP_MIN_K;
 // (distributed shared memory).
 template <int LL, int CS>
 struct FifoShared {
-  uint32_t K, types, matched, nlead;
+  uint32_t K, types, matched, nlead, p8next;
   uint32_t lg[4], lfe[4], lrl[4], lmc[4], lafter[4];
   uint64_t lgk[4];
   uint64_t ctot[2][CS];  // CTA totals of the cluster scans
@@ -748,6 +756,7 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
     }
     if (vt == 0) {
       S.matched = 0;
+      S.p8next = 0;
       S.K = 0;
       S.types = 0;
     }
@@ -1276,6 +1285,65 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             }
           }
         }
+#if MM_P8_EARLY
+        if constexpr (SMEM) {
+          // P8, early share: a warp done with its groups takes 32 receives at a
+          // time and resolves those whose result no chain can change -- the
+          // absent tuples, and the exact receives of tuples whose group has no
+          // chained wildcards (their claims are final) -- while other warps
+          // still chain.  Results are written here; recv_key records the
+          // outcome for P8's compaction (kEarlyNone, or kEarlyHit | message).
+          uint32_t nm_a = 0;
+          while (true) {
+            uint32_t c0 = 0;
+            if (lane == 0) c0 = atomicAdd(&S.p8next, 32u);
+            c0 = __shfl_sync(kFull, c0, 0);
+            if (c0 >= nr) break;
+            const uint32_t i = c0 + lane;
+            if (i >= nr) continue;
+            const uint16_t rk = ws.recv_key[i];
+            uint32_t res = kNone;
+            bool done = rk == kNone;
+            if (rk < K) {
+              const uint64_t gk = ws.keyhdr[rk] & gmsk;
+              uint32_t sl, fp;
+              slot_fp(gk, hmask, sl, fp);
+              uint32_t g = kNone32;
+              while (true) {
+                const uint32_t o = ws.table[sl];
+                if (o == kEmpty32) break;
+                if ((o >> 16) == fp && (ws.keyhdr[o & 0xFFFFu] & gmsk) == gk) {
+                  g = o & 0xFFFFu;
+                  break;
+                }
+                sl = (sl + 1) & hmask;
+              }
+              if (g != kNone32 && ws.gwc[g] == 0) {
+                done = true;
+                const uint32_t st = ws.key_start[rk], nc = ws.key_c[rk];
+                uint32_t c = 0;
+                while (c < nc && ws.wlog[st + c] < i) c++;
+                const uint32_t hd = (uint32_t)ws.recv_e[i] + c;
+                if (hd < ws.key_cnt[rk]) res = ws.by_key[st + hd];
+              }
+            }
+            if (done) {
+              a.out_rc[obase + i] = RS.cookie(i);
+              if (res != kNone) {
+                atomicOr(&ws.matched[res >> 5], 1u << (res & 31));
+                a.out_mc[obase + i] = MS.cookie(res);
+                nm_a++;
+                ws.recv_key[i] = (uint16_t)(kEarlyHit | res);
+              } else {
+                a.out_mc[obase + i] = (int64_t)MM_NO_MATCH;
+                ws.recv_key[i] = kEarlyNone;
+              }
+            }
+          }
+          for (int o = 16; o; o >>= 1) nm_a += __shfl_xor_sync(kFull, nm_a, o);
+          if (lane == 0 && nm_a) atomicAdd(&S.matched, nm_a);
+        }
+#endif
       } else if (vw == VW - 1) {
         for (uint32_t x = 0; x < W; x++) {
           const uint32_t w = ws.wl[x];
@@ -1314,6 +1382,16 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             uint32_t res = kNone;
             const int64_t rc = RS.cookie(i);
             const uint16_t rk = ws.recv_key[i];
+#if MM_P8_EARLY
+            if (SMEM && rk >= kEarlyHit && rk < kWild) {  // resolved while the chains ran
+              if (rk == kEarlyNone) {
+                fld |= 1ull << (16 * u);
+                rh[u] = RS.hdr(i);
+                rcv[u] = rc;
+              }
+              continue;
+            }
+#endif
             if (rk == kWild) {
               res = ws.recv_res[ws.recv_e[i]];
             } else if (rk != kNone) {
@@ -1515,8 +1593,14 @@ cudaError_t launch_mpi_fifo(const MpiArgs& a, const FifoLayout& L, uint8_t* gws,
   if (L.in_smem) {
     err = ensure_dyn_smem<k_mpi_fifo<256, true, 1>>((size_t)L.total);
     if (err != cudaSuccess) return err;
+    int g = grid;
+#if MM_ONCHIP_PERSIST
+    // persistent: every resident CTA slot, each serving endpoints e, e + g, ...
+    const int r = resident_ctas<k_mpi_fifo<256, true, 1>>(256, (size_t)L.total) * MM_ONCHIP_PERSIST;
+    if (g > r) g = r;
+#endif
     count_launch();
-    k_mpi_fifo<256, true, 1><<<grid, 256, (size_t)L.total, st>>>(a, L, nullptr);
+    k_mpi_fifo<256, true, 1><<<g, 256, (size_t)L.total, st>>>(a, L, nullptr);
     return cudaGetLastError();
   }
   if (L.cluster > 1) {
