@@ -153,8 +153,9 @@ int mm_push_msgs(mm_engine *e, const uint64_t *hdr, const int64_t *cookie,
  *                    cookie.  Order: MPI -- endpoint-major, queue order; the
  *                    no-wildcard levels -- every snapshot receive exactly once
  *                    in an engine-defined order (the hash-bucketed kernels
- *                    report, and keep their queues, in bucket order; the
- *                    relative order of receives with equal tuples is kept);
+ *                    report bucket by bucket, grouped by tuple; NOWILD_ORDERED
+ *                    keeps receives with equal tuples in posting order);
+ *                    residual queues keep posting / arrival order;
  *   out_msg_cookie   [out_capacity] the cookie of the message it matched, or
  *                    MM_NO_MATCH.  Either pointer may be host or device.
  *   out_capacity     length of both arrays; must cover the total snapshot
