@@ -46,6 +46,9 @@ namespace cg = cooperative_groups;
 #ifndef MM_CLUSTER_THREADS
 #define MM_CLUSTER_THREADS 512  // threads per CTA of a deep endpoint's cluster (A/B, 8 CTAs: 1024 0.094, 512 0.085 ms; no spills)
 #endif
+#ifndef MM_TABLE_CHAIN
+#define MM_TABLE_CHAIN 1  // K <= 32 chains over a CTA-built table of candidate positions (0: mask_chain)
+#endif
 #ifndef MM_P8_EARLY
 #define MM_P8_EARLY 0  // 1: P7's idle warps resolve the receives no chain can change (A/B on configs[1]: 15.8 vs 17.1 G/s -- they take issue slots from the chains)
 #endif
@@ -340,6 +343,42 @@ __device__ __forceinline__ void mask_chain(const FifoWs& ws, const uint32_t* kma
     cand = won ? l1 : l0;
     w = w2;
     r = r2;
+  }
+  if (own) ws.key_c[lane] = (uint16_t)c;
+}
+
+// mask_chain with every wildcard's candidate list position precomputed by the
+// whole CTA: E[x][k] = e_k(w_x), the exact receives of tuple k posted before
+// wildcard x, or 0xFFFF if x does not admit k.  A step is then one redux and
+// a select; the next step's E entry and its two candidate heads (for a loss
+// and for a win of this lane) load while the reduction is in flight.
+__device__ __forceinline__ void table_chain(const FifoWs& ws, const uint16_t* E, uint32_t K, uint32_t W, int lane) {
+  const bool own = (uint32_t)lane < K;
+  uint32_t st = 0, cnt = 0;
+  if (own) {
+    st = ws.key_start[lane];
+    cnt = ws.key_cnt[lane];
+  }
+  auto head = [&](uint32_t e, uint32_t p) {
+    return (own && e != 0xFFFFu && p < cnt) ? (uint32_t)ws.by_key[st + p] : 0xFFFFFFFFu;
+  };
+  uint32_t c = 0;
+  uint32_t e = E[lane];
+  uint32_t cand = head(e, e + c);
+  uint32_t en = W > 1 ? E[32 + lane] : 0xFFFFu;
+  for (uint32_t x = 0; x < W; x++) {
+    const uint32_t win = __reduce_min_sync(kFull, cand);
+    // lookahead, independent of this step's outcome
+    const uint32_t l0 = head(en, en + c), l1 = head(en, en + c + 1);
+    const uint32_t e3 = x + 2 < W ? E[(x + 2) * 32 + lane] : 0xFFFFu;
+    const bool won = win != 0xFFFFFFFFu && cand == win;
+    if (won) {
+      ws.wlog[st + c] = ws.wl[x];
+      c++;
+    }
+    if (lane == 0) ws.recv_res[x] = win == 0xFFFFFFFFu ? kNone : (uint16_t)win;
+    cand = won ? l1 : l0;
+    en = e3;
   }
   if (own) ws.key_c[lane] = (uint16_t)c;
 }
@@ -991,7 +1030,29 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
             }
           }
           bar<CS>();
+#if MM_TABLE_CHAIN
+          uint16_t* E = kpre + nch * 32;  // [W][32] after the chunk prefixes
+          if ((int64_t)nch * 32 * 6 + (int64_t)W * 64 <= (int64_t)(L.recv_res - L.gnext)) {
+            for (uint32_t t = vt; t < W * 32; t += VT) {
+              const uint32_t x = t >> 5, k = t & 31u;
+              uint16_t v = 0xFFFFu;
+              if (k < K) {
+                const uint64_t r = hdrof(x);
+                if (((ws.keyhdr[k] ^ r) & wildcard_mask(r)) == 0) {
+                  const uint32_t w = ws.wl[x], ch = w >> 5, j = w & 31u;
+                  v = (uint16_t)(kpre[ch * 32 + k] + __popc(kmask[ch * 32 + k] & ((1u << j) - 1u)));
+                }
+              }
+              E[t] = v;
+            }
+            bar<CS>();
+            if (vw == VW - 1) table_chain(ws, E, K, W, lane);
+          } else if (vw == VW - 1) {
+            mask_chain(ws, kmask, kpre, K, W, hdrof, lane);
+          }
+#else
           if (vw == VW - 1) mask_chain(ws, kmask, kpre, K, W, hdrof, lane);
+#endif
         } else if (vw == VW - 1) {
           stream_chain(ws, ws.gnext, nr, K, W, hdrof, lane);  // gnext is free here
         }
