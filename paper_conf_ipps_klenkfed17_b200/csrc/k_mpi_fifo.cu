@@ -49,6 +49,9 @@ namespace cg = cooperative_groups;
 #ifndef MM_TABLE_CHAIN
 #define MM_TABLE_CHAIN 1  // K <= 32 chains over a CTA-built table of candidate positions (0: mask_chain)
 #endif
+#ifndef MM_WILD_FIRST
+#define MM_WILD_FIRST 1  // group table built from the wildcards' keys; only tuples of those groups join (0: every tuple)
+#endif
 #ifndef MM_P8_EARLY
 #define MM_P8_EARLY 0  // 1: P7's idle warps resolve the receives no chain can change (A/B on configs[1]: 15.8 vs 17.1 G/s -- they take issue slots from the chains)
 #endif
@@ -1072,29 +1075,83 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
         const bool lead_ok = !SMEM && ws.wlog != ws.msg_key;
         const uint32_t code = __ffs(types) - 1;
         const uint64_t gmsk = (code & 1 ? ~0xFFFFFFFFull : ~0ull) & (code & 2 ? ~(0xFFFFull << 32) : ~0ull);
-        // group table: the first tuple of a group to win a slot represents it;
-        // it initialises its group entries BEFORE publishing, so members that
-        // find it may link themselves in at once (no pending state)
-        for (uint32_t k = vt; k < K; k += VT) {
-          ws.gwc[k] = 0;  // every tuple: nonzero after the wildcard pass = a representative with wildcards
-          const uint64_t gk = ws.keyhdr[k] & gmsk;
-          uint32_t s, fp;
-          slot_fp(gk, hmask, s, fp);
-          while (true) {
-            uint32_t o = ws.table[s];
-            if (o == kEmpty32) {
-              ws.gnext[k] = kNone32;
-              ws.gfirst[k] = kNone32;
-              ws.gwc[k] = 0;
-              fence<CS>();
-              o = atomicCAS(&ws.table[s], kEmpty32, (fp << 16) | k);
-              if (o == kEmpty32) break;  // k represents the group
+        auto gkey_of = [&](uint32_t eid) -> uint64_t {
+          return (eid & 0x8000u) ? (hdrof(eid & 0x7FFFu) & gmsk) : (ws.keyhdr[eid] & gmsk);
+        };
+        // (wildcards first when they are fewer than the tuples -- configs[1];
+        // else every tuple enters, the first of a group represents it --
+        // configs[4]'s thousands of wildcards over a few tuples)
+        if (MM_WILD_FIRST && W < K) {
+          // group table, wildcards first: (i) every wildcard's group key goes in
+          // as a marker (bit 15 | wildcard index); (ii) a tuple joins only if
+          // its group key is marked -- the first to replace the marker
+          // represents the group (it initialises its group entries BEFORE its
+          // CAS, so members that find it may link themselves in at once), the
+          // others link in after it; the tuples of groups without wildcards
+          // stop at their first empty slot
+          for (uint32_t x = vt; x < W; x += VT) {
+            const uint64_t rg = hdrof(x) & gmsk;
+            uint32_t s, fp;
+            slot_fp(rg, hmask, s, fp);
+            while (true) {
+              uint32_t o = ws.table[s];
+              if (o == kEmpty32) {
+                o = atomicCAS(&ws.table[s], kEmpty32, (fp << 16) | 0x8000u | x);
+                if (o == kEmpty32) break;
+              }
+              if ((o >> 16) == fp && gkey_of(o & 0xFFFFu) == rg) break;  // the group is marked already
+              s = (s + 1) & hmask;
             }
-            if ((o >> 16) == fp && (ws.keyhdr[o & 0xFFFFu] & gmsk) == gk) {
-              ws.gnext[k] = atomicExch(&ws.gnext[o & 0xFFFFu], k);  // link in after the representative
-              break;
+          }
+          bar<CS>();
+          for (uint32_t k = vt; k < K; k += VT) {
+            ws.gwc[k] = 0;  // every tuple: nonzero after the wildcard pass = a representative with wildcards
+            const uint64_t gk = ws.keyhdr[k] & gmsk;
+            uint32_t s, fp;
+            slot_fp(gk, hmask, s, fp);
+            while (true) {
+              uint32_t o = ws.table[s];
+              if (o == kEmpty32) break;  // no wildcard admits this tuple
+              if ((o >> 16) == fp && gkey_of(o & 0xFFFFu) == gk) {
+                if (o & 0x8000u) {  // still the marker: try to represent the group
+                  ws.gnext[k] = kNone32;
+                  ws.gfirst[k] = kNone32;
+                  fence<CS>();
+                  const uint32_t o2 = atomicCAS(&ws.table[s], o, (fp << 16) | k);
+                  if (o2 == o) break;  // k represents the group
+                  o = o2;             // another tuple does
+                }
+                ws.gnext[k] = atomicExch(&ws.gnext[o & 0xFFFFu], k);  // link in after the representative
+                break;
+              }
+              s = (s + 1) & hmask;
             }
-            s = (s + 1) & hmask;
+          }
+        } else {
+          // group table: the first tuple of a group to win a slot represents it;
+          // it initialises its group entries BEFORE publishing, so members that
+          // find it may link themselves in at once (no pending state)
+          for (uint32_t k = vt; k < K; k += VT) {
+            ws.gwc[k] = 0;  // every tuple: nonzero after the wildcard pass = a representative with wildcards
+            const uint64_t gk = ws.keyhdr[k] & gmsk;
+            uint32_t s, fp;
+            slot_fp(gk, hmask, s, fp);
+            while (true) {
+              uint32_t o = ws.table[s];
+              if (o == kEmpty32) {
+                ws.gnext[k] = kNone32;
+                ws.gfirst[k] = kNone32;
+                ws.gwc[k] = 0;
+                fence<CS>();
+                o = atomicCAS(&ws.table[s], kEmpty32, (fp << 16) | k);
+                if (o == kEmpty32) break;  // k represents the group
+              }
+              if ((o >> 16) == fp && (ws.keyhdr[o & 0xFFFFu] & gmsk) == gk) {
+                ws.gnext[k] = atomicExch(&ws.gnext[o & 0xFFFFu], k);  // link in after the representative
+                break;
+              }
+              s = (s + 1) & hmask;
+            }
           }
         }
         bar<CS>();
@@ -1106,8 +1163,8 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
           while (true) {
             const uint32_t o = ws.table[s];
             if (o == kEmpty32) break;
-            if ((o >> 16) == fp && (ws.keyhdr[o & 0xFFFFu] & gmsk) == rg) {
-              g = o & 0xFFFFu;
+            if ((o >> 16) == fp && gkey_of(o & 0xFFFFu) == rg) {
+              if (!(o & 0x8000u)) g = o & 0xFFFFu;  // a marker left: no tuple of the group exists
               break;
             }
             s = (s + 1) & hmask;
