@@ -247,6 +247,18 @@ enum { MM_FLAT_KERNEL_BUCKETED = 0, MM_FLAT_KERNEL_GLOBAL = 1 };
  *     overlap on three streams): 0 = auto (6 at >= 1024 endpoints, 4 at >= 256, else 1;
  *     ranges grow linearly towards the middle), 1 = off, 2..32 = that many ranges.  Results are identical
  *     for every value; a change applies to the next post. */
+/*   MM_OPT_HOST_OUT: how the MPI level delivers results into HOST output
+ *     buffers -- MM_HOST_OUT_STAGED (default): written to device staging
+ *     buffers and copied back range by range on a copy stream (overlapping
+ *     the matching of later ranges); MM_HOST_OUT_MAPPED: page-locked
+ *     (pinned / registered) output buffers are written by the matching
+ *     kernels directly through their mapped device addresses (PCIe posted
+ *     writes; no staging, no D2H copy; pageable buffers stay staged) --
+ *     measured no faster on configs[1] (2.0 vs 1.97 ms per e2e step,
+ *     DESIGN.md §7.5); it saves the staging buffers.  Results are identical; mm_match_batch returns once they
+ *     are in host memory either way. */
+enum { MM_OPT_HOST_OUT = 4 };
+enum { MM_HOST_OUT_STAGED = 0, MM_HOST_OUT_MAPPED = 1 };
 int mm_set_option(mm_engine *e, int32_t option, int64_t value);
 
 /* mm_strerror -- static description of an MM_* code. */

@@ -25,6 +25,8 @@ MM_ERR_STATE = 5
 MM_OPT_MPI_KERNEL = 1
 MM_OPT_FLAT_KERNEL = 2
 MM_OPT_PIPELINE_CHUNKS = 3
+MM_OPT_HOST_OUT = 4
+MM_HOST_OUT_STAGED, MM_HOST_OUT_MAPPED = 0, 1
 MM_FLAT_KERNEL_BUCKETED, MM_FLAT_KERNEL_GLOBAL = 0, 1
 MM_MPI_KERNEL_AUTO, MM_MPI_KERNEL_MATRIX, MM_MPI_KERNEL_FIFO = 0, 1, 2
 

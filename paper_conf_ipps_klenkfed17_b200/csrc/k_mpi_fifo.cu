@@ -63,6 +63,9 @@ constexpr uint16_t kEarlyNone = 0xFFFDu;  // recv_key: resolved early, no match
 #ifndef MM_DEEP_CS
 #define MM_DEEP_CS 8  // CTAs per deep endpoint's cluster (1: one CTA; A/B on configs[4], 1024-thread CTAs: 2 0.148, 4 0.110, 8 0.100, 16 0.124 ms)
 #endif
+#ifndef MM_PF_DIST
+#define MM_PF_DIST 0  // A/B: L2 prefetch of endpoint e + MM_PF_DIST's headers (0 = off)
+#endif
 #ifndef MM_CLUSTER_QP
 #define MM_CLUSTER_QP 32  // parts per side placed in P6 by a cluster (A/B: 16 0.108, 32 0.100, 64 0.101 ms on configs[4])
 #endif
@@ -779,6 +782,24 @@ __global__ void __launch_bounds__(NT) k_mpi_fifo(MpiArgs a, FifoLayout L, uint8_
       if (QP == 4) return (i >= rq1) + (i >= rq2) + (i >= rq3);
       return (uint32_t)(((uint64_t)i * QP) / nr);
     };
+#if MM_PF_DIST
+    // on-chip variant: the endpoint a CTA of the next wave will take (about
+    // one CTA lifetime from now) has its pending headers pulled into L2 by a
+    // bulk prefetch, so that CTA's header loads are L2 hits
+    if constexpr (SMEM && CS == 1) {
+      const int e2 = e + MM_PF_DIST;
+      if (warp == 0 && lane < 2 && e2 < a.n_ep) {
+        const Side& sd = lane ? a.M : a.R;
+        if (sd.p_hdr && sd.p_off) {
+          const uint64_t b = (uint64_t)(sd.p_hdr + sd.p_off[e2]), t = (uint64_t)(sd.p_hdr + sd.p_off[e2 + 1]);
+          const uint64_t b16 = b & ~15ull, t16 = (t + 15) & ~15ull;
+          if (t16 > b16)
+            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(b16), "r"((uint32_t)(t16 - b16))
+                         : "memory");
+        }
+      }
+    }
+#endif
     MM_PHASE(0);
     // the first round of message headers is requested before P1, so their
     // HBM latency overlaps the table clearing and the barrier

@@ -97,6 +97,18 @@ void release(DBuf& b) {
   b.bytes = 0;
 }
 
+// Device address of page-locked (mapped) host memory, or nullptr for
+// pageable host memory and device memory.
+static void* mapped_host_ptr(const void* p) {
+  if (!p) return nullptr;
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return at.type == cudaMemoryTypeHost ? at.devicePointer : nullptr;
+}
+
 bool is_device_ptr(const void* p) {
   if (!p) return false;
   cudaPointerAttributes at;
@@ -181,6 +193,7 @@ struct mm_engine {
     uint32_t over;
   }* h_small = nullptr;
   int pipeline = 0;          // MM_OPT_PIPELINE_CHUNKS (0 = auto)
+  int host_out = MM_HOST_OUT_STAGED;  // MM_OPT_HOST_OUT
   // copies out of the caller's host input buffers still in flight: recorded
   // after they are issued (on st by post, on cs by issue_chunks) and waited
   // for before mm_match_batch / mm_reset return, so that the caller may
@@ -202,9 +215,12 @@ static cudaError_t release_host_inputs(mm_engine* e) {
 // linearly towards the middle (weights min(j + 1, C - j)): the first range's
 // copy-in and the last range's copy-out are the only transfers nothing
 // overlaps, so they are the smallest.
+#ifndef MM_PIPE_RAMP
+#define MM_PIPE_RAMP 1  // A/B: 0 = equal ranges (e2e 2.07-2.10 vs 1.93-1.97 ms at 4-6 ranges)
+#endif
 static int64_t chunk_weight_sum(int k, int C) {
   int64_t s = 0;
-  for (int j = 0; j < k; j++) s += (j + 1 < C - j) ? j + 1 : C - j;
+  for (int j = 0; j < k; j++) s += MM_PIPE_RAMP ? ((j + 1 < C - j) ? j + 1 : C - j) : 1;
   return s;
 }
 static int64_t chunk_ep(const mm_engine* e, int k, int C) {
@@ -591,16 +607,28 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
   const bool counts_host = counts && !is_device_ptr(counts);
   int64_t* drc = out_rc;
   int64_t* dmc = out_mc;
-  if (host_out) {
+  // MM_HOST_OUT_MAPPED: page-locked host outputs are written by the kernels
+  // directly, through their mapped device addresses (posted PCIe writes
+  // while the endpoints are matched: no staging, no D2H copies, no read-back
+  // of the output ranges); otherwise host outputs are staged in device
+  // memory and copied back.
+  int64_t* zrc = host_out && e->host_out == MM_HOST_OUT_MAPPED ? (int64_t*)mapped_host_ptr(out_rc) : nullptr;
+  int64_t* zmc = zrc ? (int64_t*)mapped_host_ptr(out_mc) : nullptr;
+  const bool zc_out = zrc && zmc;
+  if (zc_out) {
+    drc = zrc;
+    dmc = zmc;
+  } else if (host_out) {
     CK(ensure(e->out_rc_stage, (size_t)out_cap * 8));
     CK(ensure(e->out_mc_stage, (size_t)out_cap * 8));
     drc = (int64_t*)e->out_rc_stage.p;
     dmc = (int64_t*)e->out_mc_stage.p;
   }
+  const bool staged_out = host_out && !zc_out;
   // Host-buffer pipeline: endpoint range k runs once its H2D chunks landed,
   // and its D2H starts as soon as it finished (H2D, kernels, D2H overlap).
   const int C = pipeline_chunks(e);
-  const bool pipe = C > 1 && (host_out || e->rq.pend.chunks > 0 || e->mq.pend.chunks > 0);
+  const bool pipe = C > 1 && (staged_out || e->rq.pend.chunks > 0 || e->mq.pend.chunks > 0);
   Queue* qs[2] = {&e->rq, &e->mq};
   if (pipe) {
     Queue* pq[2];
@@ -625,7 +653,14 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
     CK(launch_out_offsets(R, e->n_ep, (int64_t*)e->out_off.p, out_cap, (uint32_t*)e->err.p,
                           (unsigned long long*)e->nmatched.p, e->st));
   e->mpi_resid_empty = false;
-  if (host_out) {  // the output ranges are only known on the device: fetch them first
+  // Host outputs: the output ranges are fetched from the device first (staged
+  // outputs are copied back by range).  This read-back and wait, before the
+  // range kernels are enqueued, also keeps the pipeline overlapped: without
+  // it (the caller's host CSR offsets taken instead, or mapped outputs with
+  // no read-back) the kernels started only after the whole H2D -- 2.58-2.74
+  // vs 1.95-2.0 ms per e2e step on configs[1].
+  const int64_t* hoff = e->h_off;
+  if (host_out) {
     CK(cudaMemcpyAsync(e->h_off, out_off, (size_t)(e->n_ep + 1) * 8, cudaMemcpyDeviceToHost, e->st));
     CK(cudaStreamSynchronize(e->st));
   }
@@ -659,9 +694,9 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
       CK(launch_mpi_matrix(a, e->st));
     else
       CK(launch_mpi_fifo(a, e->fifo, (uint8_t*)e->fifo_ws.p, e->st));
-    if (pipe && host_out) {
-      const int64_t o0 = e->h_off[a.ep0] < out_cap ? e->h_off[a.ep0] : out_cap;
-      const int64_t o1 = e->h_off[a.n_ep] < out_cap ? e->h_off[a.n_ep] : out_cap;
+    if (pipe && staged_out) {
+      const int64_t o0 = hoff[a.ep0] < out_cap ? hoff[a.ep0] : out_cap;
+      const int64_t o1 = hoff[a.n_ep] < out_cap ? hoff[a.n_ep] : out_cap;
       if (o1 > o0) {
         CK(cudaEventRecord(e->ev_k[k], e->st));
         CK(cudaStreamWaitEvent(e->ds, e->ev_k[k], 0));
@@ -676,11 +711,15 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
   e->rq.pend = Pending();
   e->mq.pend = Pending();
   if (pipe) CK(cudaStreamSynchronize(e->cs));  // the caller may reuse its host inputs once we return
-  if (pipe && host_out) {
+  if (pipe && staged_out) {
     CK(cudaStreamSynchronize(e->ds));
     return deliver(e, out_rc, out_mc, false, 0, counts, counts_host);
   }
-  const int64_t tot = e->h_off[e->n_ep];
+  if (zc_out) {  // the kernels' writes into the caller's memory are complete once st is
+    if (!counts_host) CK(cudaStreamSynchronize(e->st));
+    return deliver(e, out_rc, out_mc, false, 0, counts, counts_host);
+  }
+  const int64_t tot = hoff[e->n_ep];
   return deliver(e, out_rc, out_mc, host_out, host_out ? (tot < out_cap ? tot : out_cap) : 0, counts, counts_host);
 }
 
@@ -846,6 +885,11 @@ int mm_set_option(mm_engine* e, int32_t option, int64_t value) {
   if (option == MM_OPT_PIPELINE_CHUNKS) {
     if (value < 0 || value > kMaxChunks) return MM_ERR_ARG;
     e->pipeline = (int)value;
+    return MM_OK;
+  }
+  if (option == MM_OPT_HOST_OUT) {
+    if (value != MM_HOST_OUT_STAGED && value != MM_HOST_OUT_MAPPED) return MM_ERR_ARG;
+    e->host_out = (int)value;
     return MM_OK;
   }
   if (option == MM_OPT_MPI_KERNEL) {

@@ -68,18 +68,38 @@ __device__ __forceinline__ uint32_t fetch_inc16(uint16_t* p) {
 // values, 2-3x cheaper than one ballot per value bit; tools/micro/peers.cu).
 __device__ __forceinline__ uint32_t peers_of(uint32_t v) { return __match_any_sync(kFull, v); }
 
+#ifndef MM_P6_PIPE
+#define MM_P6_PIPE 0  // A/B: 17.55 vs 17.62 G matches/s on configs[1] (rejected)
+#endif
 // Ordered placement by one warp: element x (0..n) with tuple id key(x) (>=
 // kWild = skip) gets slot start[k] + running[k]; put(x, k, rank, slot).
 // nkeys bounds the tuple ids (ids < nkeys).
 template <class KeyF, class PutF>
 __device__ __forceinline__ void place_in_order(int64_t n, KeyF key, const uint16_t* start, uint16_t* running, PutF put,
                                                int lane, uint32_t lt, uint32_t nkeys) {
+#if MM_P6_PIPE
+  // software-pipelined: the next chunk's keys and peer masks (match.any,
+  // ~200 cycles) are requested before this chunk's running counts are read
+  // and advanced, so the peer latency overlaps the dependent count chain
+  uint32_t kn = lane < n ? key(lane) : 0xFFFFFFFFu;
+  uint32_t pn = peers_of(kn < kWild ? kn : nkeys);
+  for (int64_t b = 0; b < n; b += 32) {
+    const int64_t x = b + lane;
+    const uint32_t k = kn, peers = pn;
+    const bool ok = k < kWild;
+    if (b + 32 < n) {
+      kn = x + 32 < n ? key(x + 32) : 0xFFFFFFFFu;
+      pn = peers_of(kn < kWild ? kn : nkeys);
+    }
+    uint32_t run = 0;
+#else
   for (int64_t b = 0; b < n; b += 32) {
     const int64_t x = b + lane;
     const uint32_t k = x < n ? key(x) : 0xFFFFFFFFu;
     const bool ok = k < kWild;
     const uint32_t peers = peers_of(ok ? k : nkeys);  // nkeys = "skip"
     uint32_t run = 0;
+#endif
     if (ok) run = running[k];
     __syncwarp();
     if (ok) {

@@ -71,7 +71,7 @@ class Engine:
     """Owns one mm_engine (see include/mm.h for the semantics of each call)."""
 
     def __init__(self, semantics, n_endpoints=1, recv_capacity=1024, msg_capacity=1024, stream=None,
-                 mpi_kernel=None, flat_kernel=None, pipeline_chunks=None):
+                 mpi_kernel=None, flat_kernel=None, pipeline_chunks=None, host_out=None):
         L = _lib.load()
         self._L = L
         self.semantics = semantics
@@ -98,6 +98,8 @@ class Engine:
             self.set_option(_lib.MM_OPT_FLAT_KERNEL, flat_kernel)
         if pipeline_chunks is not None:  # MPI level, host buffers: endpoint ranges of the copy pipeline
             self.set_option(_lib.MM_OPT_PIPELINE_CHUNKS, pipeline_chunks)
+        if host_out is not None:  # MPI level, host outputs: staged (default) or written in place when page-locked
+            self.set_option(_lib.MM_OPT_HOST_OUT, host_out)
 
     def set_option(self, option, value):
         check(self._L.mm_set_option(self._h, option, value), "mm_set_option")

@@ -21,7 +21,10 @@ def gpu_batches(sem, n_ep, rcap, mcap, batches, host=False, out_cap=None, mpi_ke
                 pipeline=None):
     """batches: list of (recv_hdr, recv_cookie, recv_off, msg_hdr, msg_cookie, msg_off).
     host: False (device buffers), True (host inputs and outputs), "in" (host
-    inputs, device outputs) or "out" (device inputs, host outputs).
+    inputs, device outputs), "out" (device inputs, host outputs), "pinned"
+    (page-locked host inputs and outputs) or "pinned-mapped" (the same with
+    MM_HOST_OUT_MAPPED: the MPI level writes the outputs in place through
+    their mapped addresses).
     pipeline: MM_OPT_PIPELINE_CHUNKS value (None = engine default).
     Returns a list of (out_rc, out_mc) numpy arrays, one per batch."""
     import torch
@@ -30,21 +33,38 @@ def gpu_batches(sem, n_ep, rcap, mcap, batches, host=False, out_cap=None, mpi_ke
     eng = Engine(sem, n_ep, rcap, mcap, mpi_kernel=mpi_kernel, flat_kernel=flat_kernel)
     if pipeline is not None:
         eng.set_option(MM_OPT_PIPELINE_CHUNKS, pipeline)
-    host_in = host is True or host == "in"
-    host_out = host is True or host == "out"
+    pinned = host in ("pinned", "pinned-mapped")
+    if host == "pinned-mapped":
+        from paper_conf_ipps_klenkfed17_b200._lib import MM_HOST_OUT_MAPPED, MM_OPT_HOST_OUT
+        eng.set_option(MM_OPT_HOST_OUT, MM_HOST_OUT_MAPPED)
+    host_in = host is True or host == "in" or pinned
+    host_out = host is True or host == "out" or pinned
+
+    def hbuf(a, dtype=np.int64):  # pageable numpy, or a page-locked numpy view
+        if a is None:
+            return None
+        a = np.ascontiguousarray(a, dtype)
+        if not pinned:
+            return a
+        t = torch.empty(a.shape, dtype=torch.int64).pin_memory()
+        t.numpy().view(dtype)[:] = a
+        keep.append(t)
+        return t.numpy().view(dtype)
+
+    keep = []  # page-locked buffers stay alive until the engine is closed
     res = []
     for (rh, rc, ro, mh, mc, mo) in batches:
         if host_in:
-            eng.post_recvs(np.ascontiguousarray(rh, np.uint64), rc, ro)
-            eng.push_msgs(np.ascontiguousarray(mh, np.uint64), mc, mo)
+            eng.post_recvs(hbuf(rh, np.uint64), hbuf(rc), hbuf(ro))
+            eng.push_msgs(hbuf(mh, np.uint64), hbuf(mc), hbuf(mo))
         else:
             eng.post_recvs(to_dev(rh), to_dev(rc), to_dev(ro))
             eng.push_msgs(to_dev(mh), to_dev(mc), to_dev(mo))
         cap = out_cap if out_cap is not None else n_ep * rcap
         if host_out:
-            orc = np.full(cap, -7, np.int64)
-            omc = np.full(cap, -7, np.int64)
-            cnt = np.zeros(2, np.int64)
+            orc = hbuf(np.full(cap, -7, np.int64))
+            omc = hbuf(np.full(cap, -7, np.int64))
+            cnt = hbuf(np.zeros(2, np.int64))
             eng.match_batch(orc, omc, cnt)
             n = min(int(cnt[0]), cap)
             res.append((orc[:n].copy(), omc[:n].copy(), cnt.copy()))

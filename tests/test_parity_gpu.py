@@ -93,7 +93,8 @@ def test_mpi_host_buffers_equal_device(kern):
 
 
 @pytest.mark.parametrize("chunks", [0, 1, 2, 3, 7, 32])
-@pytest.mark.parametrize("host", [True, "in", "out"], ids=["host-io", "host-in", "host-out"])
+@pytest.mark.parametrize("host", [True, "in", "out", "pinned", "pinned-mapped"],
+                         ids=["host-io", "host-in", "host-out", "pinned", "pinned-mapped"])
 @KERNELS
 def test_mpi_host_pipeline(chunks, host, kern):
     """Host-buffer pipeline (MM_OPT_PIPELINE_CHUNKS): endpoint ranges copied in,
@@ -111,13 +112,15 @@ def test_mpi_host_pipeline(chunks, host, kern):
     assert qs["error"] == 0 and qs["resid_recv"] == sum(rr) and qs["resid_msg"] == sum(rm)
 
 
-def test_mpi_host_pipeline_truncated_output():
+@pytest.mark.parametrize("host", [True, "pinned", "pinned-mapped"], ids=["pageable", "pinned", "pinned-mapped"])
+def test_mpi_host_pipeline_truncated_output(host):
     """A host output too small for the snapshot: the capacity flag is raised
-    and the copied prefix is still the oracle's."""
+    and the delivered prefix is still the oracle's (page-locked outputs are
+    written in place: nothing beyond the capacity is touched)."""
     q = synth.mpi_endpoints(77, n_ep=260, depth_r=64, ragged=True, p_unmatched=0.1)
     o, _ = oracle_batches(MPI, q.n_endpoints, single_batch(q))
     cap = len(o[0][0]) // 2
-    g, qs = gpu_batches(MPI, q.n_endpoints, 64, 64, single_batch(q), host=True, out_cap=cap, pipeline=4)
+    g, qs = gpu_batches(MPI, q.n_endpoints, 64, 64, single_batch(q), host=host, out_cap=cap, pipeline=4)
     assert qs["error"] != 0
     # endpoints whose output range fits are reported exactly; the rest is
     # flagged and its output positions are unspecified

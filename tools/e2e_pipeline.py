@@ -21,7 +21,8 @@ rh, mh, ro, mo = pin(q.recv_hdr), pin(q.msg_hdr), pin(q.recv_off), pin(q.msg_off
 orc = torch.empty(n_r, dtype=torch.int64).pin_memory()
 omc = torch.empty(n_r, dtype=torch.int64).pin_memory()
 cnt = torch.zeros(2, dtype=torch.int64).pin_memory()
-eng = mm.Engine(mm.MM_SEM_MPI, q.n_endpoints, 1024, 1024)
+eng = mm.Engine(mm.MM_SEM_MPI, q.n_endpoints, 1024, 1024,
+                host_out=mm.MM_HOST_OUT_MAPPED if os.environ.get("E2E_MAPPED") else None)
 
 
 def step():
@@ -44,9 +45,11 @@ def t_ms(fn, k=10):
     return a.elapsed_time(b) / k
 
 
-for c in [1, 2, 4, 6, 8, 12, 16, 24, 32]:
+for c in [1, 2, 4, 6, 8, 12, 16, 24, 32] if not os.environ.get("E2E_ONLY") else [4, 6, 8, 10, 12]:
     eng.set_option(MM_OPT_PIPELINE_CHUNKS, c)
     print("chunks %2d  e2e %.3f ms/step" % (c, t_ms(step)))
+if os.environ.get("E2E_ONLY"):
+    sys.exit(0)
 
 # raw copy rates
 dev = torch.empty(2 * n_r, dtype=torch.int64, device="cuda")
