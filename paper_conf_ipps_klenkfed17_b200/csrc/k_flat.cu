@@ -410,6 +410,34 @@ __global__ void k_finalize(const int64_t* n_out_src, int64_t n_out_host, const u
     user_counts[1] = b;
   }
 }
+// Device-decided tail of a bucketed no-wildcard batch (mm_engine.cu,
+// FlatTail): the overflow flag and the pair count pick the graph's
+// conditional bodies -- the global fallback + compaction, or each side's
+// compaction when it is not fully matched -- so the host never reads them
+// back; a fully matched side's residual queue is emptied here.
+__global__ void k_flat_gate(const uint32_t* over, const unsigned long long* n_matched, int64_t nr, int64_t nm,
+                            cudaGraphConditionalHandle hfb, cudaGraphConditionalHandle hr,
+                            cudaGraphConditionalHandle hm, int32_t* len_r, int32_t* len_m,
+                            unsigned long long* fallbacks) {
+  const bool fb = *over != 0;
+  const unsigned long long m = *n_matched;
+  const bool pr = !fb && (int64_t)m != nr, pm = !fb && (int64_t)m != nm;
+  cudaGraphSetConditional(hfb, fb ? 1u : 0u);
+  cudaGraphSetConditional(hr, pr ? 1u : 0u);
+  cudaGraphSetConditional(hm, pm ? 1u : 0u);
+  if (!fb && !pr) *len_r = 0;
+  if (!fb && !pm) *len_m = 0;
+  if (fb) *fallbacks += 1ull;
+}
+cudaError_t launch_flat_gate(const uint32_t* over, const unsigned long long* n_matched, int64_t nr, int64_t nm,
+                             cudaGraphConditionalHandle hfb, cudaGraphConditionalHandle hr,
+                             cudaGraphConditionalHandle hm, int32_t* len_r, int32_t* len_m,
+                             unsigned long long* fallbacks, cudaStream_t st) {
+  count_launch();
+  k_flat_gate<<<1, 1, 0, st>>>(over, n_matched, nr, nm, hfb, hr, hm, len_r, len_m, fallbacks);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_finalize(const int64_t* n_out_src, int64_t n_out_host, const unsigned long long* n_matched,
                             int64_t* counts, int64_t* user_counts, cudaStream_t st) {
   count_launch();

@@ -4,6 +4,7 @@
 // kernels of k_mpi.cu / k_flat.cu on the engine's stream.  No matching
 // arithmetic happens on the host.
 #include <nvtx3/nvToolsExt.h>
+#include <stdio.h>
 #include <stdlib.h>
 #include <string.h>
 
@@ -156,6 +157,10 @@ struct Queue {
 
 }  // namespace
 
+#ifndef MM_FLAT_TAIL
+#define MM_FLAT_TAIL 1  // device-decided tail of bucketed no-wildcard batches (0: host read-back)
+#endif
+
 struct mm_engine {
   int sem = 0;
   int n_ep = 1;
@@ -179,6 +184,27 @@ struct mm_engine {
   DBuf bh[2], bix[2], bsflag[2], bxh[2][2], bxix[2][2], bcnt, broff, bscan, bover;  // bucket regions (k_bucket.cu)
   int flat_kernel = MM_FLAT_KERNEL_BUCKETED;
   long long bucket_fallbacks = 0;
+  // Device-decided tail of bucketed no-wildcard batches (flat_tail): a CUDA
+  // graph whose conditional nodes run the global fallback and the
+  // compactions as the overflow flag and the pair count decide on the
+  // device, so the batch needs no host read-back.  Instantiated graphs are
+  // cached by everything their launches capture (TailKey).
+  struct TailKey {
+    FlatArgs a;
+    const void* ptr[24];
+    int64_t val[8];
+  };
+  struct TailGraph {
+    TailKey key;
+    cudaGraphExec_t exec = nullptr;
+    long long stamp = 0;
+  };
+  static constexpr int kTailCache = 4;
+  TailGraph tails[kTailCache];
+  long long tail_clock = 0;
+  cudaStream_t gs = nullptr;  // capture stream
+  DBuf fb_dev;                // fallbacks taken by device-decided tails
+  int tail_mode = 1;          // MM_FLAT_TAIL A/B: 0 = host read-back of the overflow flag and the pair count
   Timer timer;
   long long launches = 0;
   // host-buffer pipeline: H2D copies on cs, D2H copies on ds, chunk kernels on st
@@ -245,10 +271,17 @@ struct LaunchScope {
   }
 };
 
-#define CK(x)                                   \
-  do {                                          \
-    cudaError_t _e = (x);                       \
-    if (_e != cudaSuccess) return MM_ERR_CUDA;  \
+// MM_DEBUG=1 in the environment: every failing CUDA call is reported on
+// stderr (file:line and the CUDA error) before MM_ERR_CUDA is returned.
+static int ck_fail(cudaError_t e, int line) {
+  static const bool dbg = getenv("MM_DEBUG") != nullptr;
+  if (dbg) fprintf(stderr, "mm_engine.cu:%d: %s\n", line, cudaGetErrorString(e));
+  return MM_ERR_CUDA;
+}
+#define CK(x)                                               \
+  do {                                                      \
+    cudaError_t _e = (x);                                   \
+    if (_e != cudaSuccess) return ck_fail(_e, __LINE__);    \
   } while (0)
 
 static Side make_side(mm_engine* e, Queue& q, int64_t cap) {
@@ -308,6 +341,9 @@ int mm_destroy(mm_engine* e) {
   if (e->ev_st) cudaEventDestroy(e->ev_st);
   if (e->ev_in_st) cudaEventDestroy(e->ev_in_st);
   if (e->ev_in_cs) cudaEventDestroy(e->ev_in_cs);
+  for (auto& t : e->tails)
+    if (t.exec) cudaGraphExecDestroy(t.exec);
+  if (e->gs) cudaStreamDestroy(e->gs);
   if (e->cs) cudaStreamDestroy(e->cs);
   if (e->ds) cudaStreamDestroy(e->ds);
   if (e->h_off) cudaFreeHost(e->h_off);
@@ -328,7 +364,7 @@ int mm_destroy(mm_engine* e) {
                   &e->owner, &e->rcnt, &e->mcnt, &e->tkey, &e->tval, &e->fifo_ws,
                   &e->bh[0], &e->bh[1], &e->bix[0], &e->bix[1], &e->bsflag[0], &e->bsflag[1], &e->bcnt,
                   &e->broff, &e->bscan, &e->bover, &e->bxh[0][0], &e->bxh[0][1], &e->bxh[1][0], &e->bxh[1][1],
-                  &e->bxix[0][0], &e->bxix[0][1], &e->bxix[1][0], &e->bxix[1][1]};
+                  &e->bxix[0][0], &e->bxix[0][1], &e->bxix[1][0], &e->bxix[1][1], &e->fb_dev};
   for (DBuf* b : bufs) release(*b);
   delete e;
   return MM_OK;
@@ -370,12 +406,18 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
   bool ok = ensure(e->out_off, (size_t)(n_endpoints + 1) * 8) == cudaSuccess &&
             ensure(e->counts_dev, 16) == cudaSuccess && ensure(e->nmatched, 8) == cudaSuccess &&
             ensure(e->err, 4) == cudaSuccess && ensure(e->info, sizeof(SnapInfo)) == cudaSuccess;
+  // (every level: host inputs are copied out of the caller's buffers)
+  ok = ok && cudaEventCreateWithFlags(&e->ev_in_st, cudaEventDisableTiming) == cudaSuccess &&
+       cudaEventCreateWithFlags(&e->ev_in_cs, cudaEventDisableTiming) == cudaSuccess;
+  if (ok && semantics != MM_SEM_MPI) {
+    ok = cudaStreamCreateWithFlags(&e->gs, cudaStreamNonBlocking) == cudaSuccess &&
+         ensure(e->fb_dev, 8) == cudaSuccess && cudaMemset(e->fb_dev.p, 0, 8) == cudaSuccess;
+    e->tail_mode = MM_FLAT_TAIL;
+  }
   if (ok && semantics == MM_SEM_MPI) {
     ok = cudaStreamCreateWithFlags(&e->cs, cudaStreamNonBlocking) == cudaSuccess &&
          cudaStreamCreateWithFlags(&e->ds, cudaStreamNonBlocking) == cudaSuccess &&
          cudaEventCreateWithFlags(&e->ev_st, cudaEventDisableTiming) == cudaSuccess &&
-         cudaEventCreateWithFlags(&e->ev_in_st, cudaEventDisableTiming) == cudaSuccess &&
-         cudaEventCreateWithFlags(&e->ev_in_cs, cudaEventDisableTiming) == cudaSuccess &&
          cudaMallocHost(&e->h_off, (size_t)(n_endpoints + 1) * 8) == cudaSuccess;
     for (int k = 0; ok && k < kMaxChunks; k++)
       ok = cudaEventCreateWithFlags(&e->ev_k[k], cudaEventDisableTiming) == cudaSuccess &&
@@ -723,6 +765,136 @@ static int match_mpi(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out
   return deliver(e, out_rc, out_mc, host_out, host_out ? (tot < out_cap ? tot : out_cap) : 0, counts, counts_host);
 }
 
+extern "C++" {
+// Capture the launches f(stream) into graph g (appended as root nodes); the
+// captured launches are not counted as executed (a conditional body may not
+// run).
+template <class F>
+static cudaError_t capture_into(cudaStream_t gs, cudaGraph_t g, F&& f) {
+  cudaError_t err = cudaStreamBeginCaptureToGraph(gs, g, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed);
+  if (err != cudaSuccess) return err;
+  const long long lc = launch_count();
+  const cudaError_t fe = f(gs);
+  launch_count() = lc;
+  cudaGraph_t out = g;
+  err = cudaStreamEndCapture(gs, &out);
+  return fe != cudaSuccess ? fe : err;
+}
+
+// Append an IF node (after dep) whose body holds the launches of f.
+template <class F>
+static cudaError_t add_if(cudaStream_t gs, cudaGraph_t g, cudaGraphNode_t dep, cudaGraphConditionalHandle h,
+                          cudaGraphNode_t* node, F&& f) {
+  cudaGraphNodeParams p = {};
+  p.type = cudaGraphNodeTypeConditional;
+  p.conditional.handle = h;
+  p.conditional.type = cudaGraphCondTypeIf;
+  p.conditional.size = 1;
+  cudaError_t err = cudaGraphAddNode(node, g, &dep, 1, &p);
+  if (err != cudaSuccess) return err;
+  return capture_into(gs, p.conditional.phGraph_out[0], f);
+}
+
+}  // extern "C++"
+
+// The tail of a bucketed no-wildcard batch, decided on the device (one
+// graph launch, no host read-back): gate -> IF(overflow) {pair count reset,
+// global fallback -- the sort-and-rank over all 64 header bits, or the hash
+// table --, both compactions} -> IF(receives partly matched) {slot flags,
+// compaction} -> IF(messages partly matched) {slot flags, compaction}; a
+// fully matched side's residual queue is emptied by the gate.
+static int flat_tail(mm_engine* e, const FlatArgs& a, const BucketScratch& bs, bool ordered, const int64_t res[2],
+                     const int64_t ns[2]) {
+  Queue* qs[2] = {&e->rq, &e->mq};
+  SortScratch ss;
+  for (int b = 0; b < 2; b++) {
+    ss.key[b] = (uint64_t*)e->skey[b].p;
+    ss.val[b] = (uint32_t*)e->sval[b].p;
+  }
+  ss.rid = (uint32_t*)e->rid.p;
+  ss.run_start = (uint32_t*)e->run_start.p;
+  ss.run_rc = (uint32_t*)e->run_rc.p;
+  ss.part = (uint32_t*)e->part.p;
+  ss.scan = (unsigned long long*)e->scan.p;
+  HashScratch hs;
+  hs.owner = (uint32_t*)e->owner.p;
+  hs.rcnt = (uint32_t*)e->rcnt.p;
+  hs.mcnt = (uint32_t*)e->mcnt.p;
+  hs.tkey = (unsigned long long*)e->tkey.p;
+  hs.tval = (uint32_t*)e->tval.p;
+  hs.T = next_pow2(2 * a.nr < 1024 ? 1024 : 2 * a.nr);
+  mm_engine::TailKey key;
+  memset(&key, 0, sizeof(key));
+  key.a = a;
+  const void* ptrs[] = {bs.bcnt, bs.ix[0], bs.ix[1], bs.sflag[0], bs.sflag[1], bs.overflow,
+                        e->rq.hdr[e->rq.cur ^ 1].p, e->rq.cookie[e->rq.cur ^ 1].p, e->rq.len[e->rq.cur ^ 1].p,
+                        e->mq.hdr[e->mq.cur ^ 1].p, e->mq.cookie[e->mq.cur ^ 1].p, e->mq.len[e->mq.cur ^ 1].p,
+                        e->scan.p, ss.key[0], ss.key[1], ss.val[0], ss.val[1], ss.rid, ss.run_start, ss.run_rc,
+                        ss.part, hs.owner, hs.tkey, e->fb_dev.p};
+  static_assert(sizeof(ptrs) == sizeof(key.ptr), "TailKey pointers");
+  memcpy(key.ptr, ptrs, sizeof(ptrs));
+  const int64_t vals[] = {res[0], res[1], ns[0], ns[1], (int64_t)bs.B, ordered ? 1 : 0, hs.T, 0};
+  memcpy(key.val, vals, sizeof(vals));
+  mm_engine::TailGraph* t = nullptr;
+  for (auto& c : e->tails)
+    if (c.exec && memcmp(&c.key, &key, sizeof(key)) == 0) t = &c;
+  if (!t) {  // build: evict the least recently used entry
+    t = &e->tails[0];
+    for (auto& c : e->tails)
+      if (!c.exec || c.stamp < t->stamp) t = &c;
+    if (t->exec) cudaGraphExecDestroy(t->exec);
+    t->exec = nullptr;
+    cudaGraph_t g;
+    CK(cudaGraphCreate(&g, 0));
+    cudaGraphConditionalHandle h[3];
+    cudaError_t err = cudaSuccess;
+    for (int i = 0; i < 3 && err == cudaSuccess; i++) err = cudaGraphConditionalHandleCreate(&h[i], g, 0, cudaGraphCondAssignDefault);
+    if (err == cudaSuccess)
+      err = capture_into(e->gs, g, [&](cudaStream_t st) {
+        return launch_flat_gate(bs.overflow, a.n_matched, a.nr, a.nm, h[0], h[1], h[2],
+                                (int32_t*)e->rq.len[e->rq.cur ^ 1].p, (int32_t*)e->mq.len[e->mq.cur ^ 1].p,
+                                (unsigned long long*)e->fb_dev.p, st);
+      });
+    cudaGraphNode_t prev = nullptr;
+    size_t nn = 1;
+    if (err == cudaSuccess) err = cudaGraphGetRootNodes(g, &prev, &nn);
+    auto compact = [&](int i, const uint8_t* flags, cudaStream_t st) {
+      Queue& q = *qs[i];
+      const int nb = q.cur ^ 1;
+      return run_compact(i ? a.M : a.R, res[i], ns[i], flags, (uint64_t*)q.hdr[nb].p, (int64_t*)q.cookie[nb].p,
+                         (int32_t*)q.len[nb].p, (uint32_t*)e->scan.p, st);
+    };
+    cudaGraphNode_t n0, n1, n2;
+    if (err == cudaSuccess)
+      err = add_if(e->gs, g, prev, h[0], &n0, [&](cudaStream_t st) {
+        cudaError_t r = cudaMemsetAsync(a.n_matched, 0, 8, st);
+        if (r == cudaSuccess) r = ordered ? run_sort_rank(a, 0ull, ~0ull, ss, st) : run_hash(a, hs, st);
+        if (r == cudaSuccess) r = compact(0, a.rflag, st);
+        if (r == cudaSuccess) r = compact(1, a.mflag, st);
+        return r;
+      });
+    for (int i = 0; i < 2 && err == cudaSuccess; i++)
+      err = add_if(e->gs, g, i ? n1 : n0, h[1 + i], i ? &n2 : &n1, [&](cudaStream_t st) {
+        uint8_t* fl = i ? a.mflag : a.rflag;
+        cudaError_t r = run_slot_flags(bs, i, fl, st);
+        if (r == cudaSuccess) r = compact(i, fl, st);
+        return r;
+      });
+    if (err == cudaSuccess) err = cudaGraphInstantiate(&t->exec, g, 0);
+    cudaGraphDestroy(g);
+    if (err != cudaSuccess) {
+      t->exec = nullptr;
+      cudaGetLastError();
+      return MM_ERR_CUDA;
+    }
+    t->key = key;
+  }
+  t->stamp = ++e->tail_clock;
+  count_launch();  // the gate; the bodies run only when it says so
+  CK(cudaGraphLaunch(t->exec, e->st));
+  return MM_OK;
+}
+
 static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t out_cap, int64_t* counts) {
   const bool host_out = !is_device_ptr(out_rc) || !is_device_ptr(out_mc);
   const bool counts_host = counts && !is_device_ptr(counts);
@@ -787,6 +959,27 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
     e->timer.begin(e->st);
     CK(run_bucketed(a, ordered, bs, e->st));
     e->timer.end(e->st);
+    if (e->tail_mode) {
+      const int64_t res[2] = {info.rres, info.mres}, ns[2] = {nr, nm};
+      const int tr = flat_tail(e, a, bs, ordered, res, ns);
+      if (tr != MM_OK) return tr;
+      CK(launch_finalize(nullptr, nr, (const unsigned long long*)e->nmatched.p, (int64_t*)e->counts_dev.p,
+                         counts && !counts_host ? counts : nullptr, e->st));
+      // the residual sizes are known again only if the pair count comes back
+      // anyway (host outputs or host counts: the call synchronises)
+      const bool back = host_out || counts_host;
+      if (back) CK(cudaMemcpyAsync(&e->h_small->matched, e->nmatched.p, 8, cudaMemcpyDeviceToHost, e->st));
+      const int dr = deliver(e, out_rc, out_mc, host_out, nr < out_cap ? nr : out_cap, counts, counts_host);
+      Queue* qs2[2] = {&e->rq, &e->mq};
+      const int64_t ns2[2] = {nr, nm};
+      for (int i = 0; i < 2; i++) {
+        qs2[i]->cur ^= 1;
+        qs2[i]->pend = Pending();
+        qs2[i]->resid_host = back ? ns2[i] - (int64_t)e->h_small->matched : ns2[i];
+        qs2[i]->resid_exact = back;
+      }
+      return dr;
+    }
     CK(cudaMemcpyAsync(&e->h_small->over, e->bover.p, 4, cudaMemcpyDeviceToHost, e->st));
     CK(cudaMemcpyAsync(&e->h_small->matched, e->nmatched.p, 8, cudaMemcpyDeviceToHost, e->st));
     CK(cudaStreamSynchronize(e->st));
@@ -925,7 +1118,9 @@ int mm_query(mm_engine* e, int64_t* vals) {
   vals[MM_Q_KERNEL_NS] = e->timer.ns;
   vals[MM_Q_KERNEL_RUNS] = e->timer.runs;
   vals[MM_Q_LAUNCHES] = e->launches;
-  vals[MM_Q_FALLBACKS] = e->bucket_fallbacks;
+  unsigned long long fbd = 0;
+  if (e->fb_dev.p) CK(cudaMemcpy(&fbd, e->fb_dev.p, 8, cudaMemcpyDeviceToHost));
+  vals[MM_Q_FALLBACKS] = e->bucket_fallbacks + (int64_t)fbd;
   if (e->sem != MM_SEM_MPI) {
     e->rq.resid_host = rsum;
     e->mq.resid_host = msum;

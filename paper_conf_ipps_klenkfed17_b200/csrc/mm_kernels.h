@@ -96,6 +96,15 @@ struct HashScratch {
 };
 cudaError_t run_hash(const FlatArgs& a, const HashScratch& h, cudaStream_t st);
 
+// Gate of the device-decided tail of a bucketed batch (one thread): sets the
+// graph's conditional handles (fallback / partly matched receives / partly
+// matched messages), empties the residual queue of a fully matched side and
+// counts fallbacks.
+cudaError_t launch_flat_gate(const uint32_t* over, const unsigned long long* n_matched, int64_t nr, int64_t nm,
+                             cudaGraphConditionalHandle hfb, cudaGraphConditionalHandle hr,
+                             cudaGraphConditionalHandle hm, int32_t* len_r, int32_t* len_m,
+                             unsigned long long* fallbacks, cudaStream_t st);
+
 // Both no-wildcard levels, hash-bucketed (k_bucket.cu): one-pass partition
 // into fixed-capacity bucket regions + one CTA per bucket.  Sets *overflow if
 // a bucket does not fit (the caller then falls back to run_sort_rank /

@@ -416,12 +416,17 @@ def test_ordered_wide_keys_and_wildcard_values(flat):
 
 
 @pytest.mark.parametrize("seed", range(3))
+@pytest.mark.parametrize("host", [False, True], ids=["dev", "host"])
 @FLAT
-def test_ordered_multibatch(seed, flat):
+def test_ordered_multibatch(seed, flat, host):
+    """Three batches with residual queues.  Device buffers: the bucketed
+    batches' tails are decided on the device (no read-back; the next batch
+    reads the residual sizes first); host buffers: the pair count comes back
+    with the outputs."""
     rng = np.random.default_rng(seed)
     q = synth.nowild_pairs(seed + 3, n=30000, n_src=300, n_tag=4, p_unmatched=0.3)
     batches = split_batches(q, 3, rng)
-    g, _ = gpu_batches(ORD, 1, 60000, 60000, batches, flat_kernel=flat)
+    g, _ = gpu_batches(ORD, 1, 60000, 60000, batches, flat_kernel=flat, host=host)
     o, _ = oracle_batches(ORD, 1, batches)
     assert_same_pairs(g, o)
 
@@ -432,9 +437,46 @@ def test_ordered_all_same_key(flat):
     rh = synth.pack(np.full(n, 4), np.full(n, 2))
     mh = synth.pack(np.full(n - 17, 4), np.full(n - 17, 2))
     b = [(rh, None, np.array([0, n]), mh, None, np.array([0, n - 17]))]
-    g, _ = gpu_batches(ORD, 1, n, n, b, flat_kernel=flat)
+    g, qs = gpu_batches(ORD, 1, n, n, b, flat_kernel=flat)
     o, _ = oracle_batches(ORD, 1, b)
     assert_same_pairs(g, o)
+    assert flat != 0 or qs["fallbacks"] == 1  # the bucketed run overflowed: global fallback
+
+
+@pytest.mark.parametrize("sem", [ORD, UNO], ids=["ordered", "unordered"])
+@pytest.mark.parametrize("host", [False, True], ids=["dev", "host"])
+def test_bucket_fallback_between_bucketed_batches(sem, host):
+    """Batch 1 overflows the buckets (one tuple repeated thousands of times:
+    the global fallback and its compaction run inside the device-decided
+    tail), batch 2 is bucketed again on the residual queues of batch 1,
+    batch 3 overflows again: per batch identical to the oracle (ordered) /
+    valid and maximal (unordered)."""
+    rng = np.random.default_rng(4)
+    seq = [0, 0]  # cookies: global receive / message ids
+
+    def batch(n, hot):
+        src = rng.integers(0, 1 << 20, n)
+        tag = rng.integers(0, 8, n)
+        if hot:
+            src[: n // 2] = 5
+            tag[: n // 2] = 1
+        rh = synth.pack(src, tag)
+        mh = rh[rng.permutation(n)][: n - 13]
+        rc = np.arange(seq[0], seq[0] + n, dtype=np.int64)
+        mc = np.arange(seq[1], seq[1] + n - 13, dtype=np.int64)
+        seq[0] += n
+        seq[1] += n - 13
+        return (rh, rc, np.array([0, n]), mh, mc, np.array([0, n - 13]))
+    b = [batch(9000, True), batch(7000, False), batch(8000, True)]
+    g, qs = gpu_batches(sem, 1, 30000, 30000, b, flat_kernel=0, host=host)
+    assert qs["fallbacks"] == 2
+    if sem == ORD:
+        o, _ = oracle_batches(ORD, 1, b)
+        assert_same_pairs(g, o)
+    else:
+        rh = np.concatenate([x[0] for x in b])
+        mh = np.concatenate([x[3] for x in b])
+        check_unordered_per_batch(g, b, rh, mh)
 
 
 def test_ordered_long_runs_stay_on_chip():
@@ -492,12 +534,13 @@ def check_min(q):
 
 
 @pytest.mark.parametrize("seed", range(3))
+@pytest.mark.parametrize("host", [False, True], ids=["dev", "host"])
 @FLAT
-def test_unordered_multibatch(seed, flat):
+def test_unordered_multibatch(seed, flat, host):
     rng = np.random.default_rng(seed)
     q = synth.nowild_pairs(seed + 7, n=20000, n_src=200, n_tag=3, p_unmatched=0.3)
     batches = split_batches(q, 3, rng)
-    g, _ = gpu_batches(UNO, 1, 40000, 40000, batches, flat_kernel=flat)
+    g, _ = gpu_batches(UNO, 1, 40000, 40000, batches, flat_kernel=flat, host=host)
     # across all batches: every pair has equal tuples, every element used once,
     # and the total per tuple is min(#recv, #msg) of the whole input
     rc = np.concatenate([x[0] for x in g])
