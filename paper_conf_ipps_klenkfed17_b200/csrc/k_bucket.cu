@@ -42,24 +42,26 @@ struct SnapRead {
   __device__ __forceinline__ uint64_t hdr(int64_t u) const { return u < resid ? q[u] : p[u - resid]; }
 };
 
-// Buckets: B = 2^nb with at most kAvgSide elements of the larger side per
-// bucket on average; each bucket owns a fixed region of kSideCap slots per
-// side (a bucket above it -- heavily repeated tuples -- flags an overflow).
-constexpr int kAvgSide = 512;
-constexpr uint32_t kSideCap = 1536;
+// Buckets: B = 2^nb with at most `avg` elements of the larger side per
+// bucket on average; each bucket owns a fixed region of 3 avg slots per side
+// (a bucket above it -- heavily repeated tuples -- flags an overflow).  The
+// geometry is per level (bucket_avg): NOWILD_ORDERED 256 elements per side
+// with 128-thread CTAs, six per SM; NOWILD_UNORDERED 512 with 256-thread
+// CTAs, three per SM (A/B).
+int bucket_avg(bool ordered) { return ordered ? 256 : 512; }
 
-int bucket_bits_for(int64_t n_side) {
+int bucket_bits_for(int64_t n_side, int avg) {
   int nb = 1;
-  while (nb < 30 && ((int64_t)1 << nb) * kAvgSide < n_side) nb++;
+  while (nb < 30 && ((int64_t)1 << nb) * avg < n_side) nb++;
   return nb;
 }
-int64_t bucket_count(int64_t n_side) { return (int64_t)1 << bucket_bits_for(n_side); }
+int64_t bucket_count(int64_t n_side, int avg) { return (int64_t)1 << bucket_bits_for(n_side, avg); }
 
 // ------------------------------------------------------------- partition
 // MSD passes over the bucket id b = bucket_of(hdr) (nb bits): pass 0 reads
 // the snapshot and splits each side by the top bits of b, every later pass
 // splits each region of the previous one by the next bits; the last pass
-// writes the buckets' kSideCap-slot regions.  Every region has a fixed
+// writes the buckets' 3 avg-slot regions.  Every region has a fixed
 // capacity (the expected size x 1.25 + 256 on intermediate levels), so a
 // pass needs no histogram pass and no scan: a tile of kPassTile elements
 // ranks its elements per digit with shared-memory atomics, reserves each
@@ -83,9 +85,9 @@ constexpr int kPassItems = MM_PASS_ITEMS;
 constexpr int kPassTile = kPassThreads * kPassItems;  // 4096
 constexpr int kPassMaxKeys = 1024;                    // digits per tile (pass 0: both sides' digits)
 
-PartPlan part_plan(int64_t n_side) {
+PartPlan part_plan(int64_t n_side, int avg) {
   PartPlan pl{};
-  pl.nb = bucket_bits_for(n_side);
+  pl.nb = bucket_bits_for(n_side, avg);
   // pass 0 takes at most 8 bits (2 x 256 keys per tile), later passes at most 10
   int rest = pl.nb;
   int bits[kMaxPasses];
@@ -110,7 +112,7 @@ PartPlan part_plan(int64_t n_side) {
     pl.shift[i] = pl.nb - done;
     pl.children[i] = (int64_t)1 << done;  // per side
     if (i == np - 1) {
-      pl.cap[i] = kSideCap;
+      pl.cap[i] = 3 * avg;
     } else {
       const int64_t expect = (n_side + pl.children[i] - 1) / pl.children[i];
       pl.cap[i] = (expect + expect / 4 + 256 + 15) / 16 * 16;
@@ -268,9 +270,10 @@ __global__ void __launch_bounds__(kPassThreads, MM_PASS_MINB) k_part_pass(PassAr
 // Output offsets of the buckets: exclusive scan of the receive counts.
 struct BucketCountIn {
   const uint32_t* cnt;
+  uint32_t cap;
   __device__ __forceinline__ uint32_t operator()(int64_t b) const {
     const uint32_t c = cnt[b];
-    return c < kSideCap ? c : kSideCap;
+    return c < cap ? c : cap;
   }
 };
 struct BucketOffOut {
@@ -303,35 +306,36 @@ struct BucketOffOut {
 //     written coalesced at the bucket's output offset in group order, and a
 //     matched byte per bucket slot (coalesced) serves a later compaction.
 // O(1) shared-memory work per element (F: O(group size)), 7 barriers.
-constexpr int kMatchK = 2048;  // receives + messages of one bucket on chip
-constexpr int kMatchThreads = 256;
 constexpr uint32_t kNone32 = 0xFFFFFFFFu;
-constexpr uint32_t kMatchH = 4096;  // table slots (>= 2 kMatchK)
 
-// 64 KB: three CTAs per SM.  Arrays that die with a phase share space with
-// arrays that start later.
+// Shared memory of one bucket of up to K = 4 avg elements (receives +
+// messages) and H = 8 avg table slots: 32 B per element (avg 512: 64 KB,
+// three CTAs per SM; avg 256: 32 KB, six).  Arrays that die with a phase
+// share space with arrays that start later.
+template <int K, int H, int NT>
 struct MatchSmem {
   union {
-    uint64_t hdr[kMatchK];  // A..B: headers (table keys)
+    uint64_t hdr[K];  // A..B: headers (table keys)
     struct {
-      uint32_t aidx[kMatchK];  // E..F: snapshot index of each grouped element
-      uint16_t srt[kMatchK];   // F..G: every group in snapshot order
+      uint32_t aidx[K];  // E..F: snapshot index of each grouped element
+      uint16_t srt[K];   // F..G: every group in snapshot order
     };
   };
   union {
-    uint32_t table[kMatchH];  // A..B: (fingerprint << 16) | representative element
-    uint16_t area[kMatchK];   // E..F: receives [0, nr) then messages [nr, n), grouped by tuple
+    uint32_t table[H];  // A..B: (fingerprint << 16) | representative element
+    uint16_t area[K];   // E..F: receives [0, nr) then messages [nr, n), grouped by tuple
   };
-  uint32_t idx[kMatchK];      // snapshot index
-  uint16_t sid[kMatchH];      // B..C: slot -> dense tuple id
-  uint16_t tup[kMatchK];      // B: element -> slot; C..: tuple id
-  uint16_t pos[kMatchK];      // C..E: position among its side's equal tuples
-  uint32_t pre[kMatchK + 1];  // C: packed counts (#recv | #msg << 16); D..: packed group starts, pre[T] = totals
-  uint32_t wsum[kMatchThreads / 32];
+  uint32_t idx[K];      // snapshot index
+  uint16_t sid[H];      // B..C: slot -> dense tuple id
+  uint16_t tup[K];      // B: element -> slot; C..: tuple id
+  uint16_t pos[K];      // C..E: position among its side's equal tuples
+  uint32_t pre[K + 1];  // C: packed counts (#recv | #msg << 16); D..: packed group starts, pre[T] = totals
+  uint32_t wsum[NT / 32];
   uint32_t ntup;
   uint32_t nmatch;
 };
-static_assert(sizeof(MatchSmem) <= 74 * 1024, "three CTAs per SM");
+static_assert(sizeof(MatchSmem<2048, 4096, 256>) <= 74 * 1024, "avg 512: three CTAs per SM");
+static_assert(sizeof(MatchSmem<1024, 2048, 128>) <= 37 * 1024, "avg 256: six CTAs per SM");
 
 struct MatchArgs {
   FlatArgs a;
@@ -360,11 +364,13 @@ __device__ unsigned long long g_bucket_cycles[16];
   } while (0)
 #endif
 
-template <bool ORDERED>
-__global__ void __launch_bounds__(kMatchThreads, 3) k_bucket_match(MatchArgs ma) {
+template <bool ORDERED, int AVG, int NT, int MINB>
+__global__ void __launch_bounds__(NT, MINB) k_bucket_match(MatchArgs ma) {
+  constexpr int kMatchK = 4 * AVG;            // receives + messages of one bucket on chip
+  constexpr uint32_t kMatchH = 8 * AVG;       // table slots (>= 2 kMatchK)
+  constexpr uint32_t kSideCap = 3 * AVG;      // region slots per side
   extern __shared__ __align__(16) uint8_t smem_raw[];
-  MatchSmem& sm = *reinterpret_cast<MatchSmem*>(smem_raw);
-  constexpr int NT = kMatchThreads;
+  auto& sm = *reinterpret_cast<MatchSmem<kMatchK, kMatchH, NT>*>(smem_raw);
   constexpr int PER = kMatchK / NT;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t lt = lanemask_lt();
@@ -595,10 +601,10 @@ static uint32_t persistent_grid(int threads, size_t smem, uint32_t B) {
 }
 
 // Largest allocation any batch of at most n_side elements per side needs.
-PartPlan part_plan_alloc(int64_t n_side) {
-  PartPlan m = part_plan(n_side);
+PartPlan part_plan_alloc(int64_t n_side, int avg) {
+  PartPlan m = part_plan(n_side, avg);
   for (int nb = 1; nb < m.nb; nb++) {
-    const PartPlan p = part_plan(((int64_t)1 << nb) * kAvgSide);
+    const PartPlan p = part_plan(((int64_t)1 << nb) * avg, avg);
     for (int j = 0; j < 2; j++)
       if (p.scratch_slots[j] > m.scratch_slots[j]) m.scratch_slots[j] = p.scratch_slots[j];
     if (p.cnt_total > m.cnt_total) m.cnt_total = p.cnt_total;
@@ -606,8 +612,23 @@ PartPlan part_plan_alloc(int64_t n_side) {
   return m;
 }
 
+// One bucket geometry's matching kernel: avg elements per side and bucket,
+// NT threads, MINB CTAs per SM.
+template <bool ORDERED, int AVG, int NT, int MINB>
+static cudaError_t launch_bucket_match(const MatchArgs& ma, uint32_t B, cudaStream_t st) {
+  constexpr auto kern = k_bucket_match<ORDERED, AVG, NT, MINB>;
+  const size_t smem = sizeof(MatchSmem<4 * AVG, 8 * AVG, NT>);
+  cudaError_t err = ensure_dyn_smem<kern>(smem);
+  if (err != cudaSuccess) return err;
+  count_launch();
+  kern<<<persistent_grid<kern>(NT, smem, B), NT, smem, st>>>(ma);
+  return cudaGetLastError();
+}
+
 cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cudaStream_t st) {
-  const PartPlan pl = part_plan(a.nr > a.nm ? a.nr : a.nm);
+  const int avg = bucket_avg(ordered);
+  const PartPlan pl = part_plan(a.nr > a.nm ? a.nr : a.nm, avg);
+  s.side_cap = 3 * avg;
   const int nb = pl.nb;
   const uint32_t B = 1u << nb;
   s.plan = pl;
@@ -652,7 +673,8 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cuda
     }
     if ((err = cudaGetLastError()) != cudaSuccess) return err;
   }
-  if ((err = scan_apply<uint32_t>(BucketCountIn{s.bcnt}, (int64_t)B, s.scan, BucketOffOut{s.roff, (int64_t)B}, st)) !=
+  if ((err = scan_apply<uint32_t>(BucketCountIn{s.bcnt, (uint32_t)s.side_cap}, (int64_t)B, s.scan,
+                                  BucketOffOut{s.roff, (int64_t)B}, st)) !=
       cudaSuccess)
     return err;
   MatchArgs ma;
@@ -667,35 +689,27 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cuda
   ma.sflag[1] = s.sflag[1];
   ma.overflow = s.overflow;
   ma.B = B;
-  const size_t smem = sizeof(MatchSmem);
-  count_launch();
-  if (ordered) {
-    if ((err = ensure_dyn_smem<k_bucket_match<true>>(smem)) != cudaSuccess) return err;
-    k_bucket_match<true><<<persistent_grid<k_bucket_match<true>>(kMatchThreads, smem, B), kMatchThreads, smem, st>>>(ma);
-  } else {
-    if ((err = ensure_dyn_smem<k_bucket_match<false>>(smem)) != cudaSuccess) return err;
-    k_bucket_match<false><<<persistent_grid<k_bucket_match<false>>(kMatchThreads, smem, B), kMatchThreads, smem, st>>>(
-        ma);
-  }
-  return cudaGetLastError();
+  if (ordered) return launch_bucket_match<true, 256, 128, 6>(ma, B, st);
+  return launch_bucket_match<false, 512, 256, 3>(ma, B, st);
 }
 
 // Partly matched side: the bucket slots' matched bytes scattered to snapshot
 // order, so that the compaction keeps the residual queue in posting / arrival
 // order (run_compact).
 __global__ void k_slot_flags(const uint32_t* cnt, const uint32_t* ix, const uint8_t* sflag, int64_t nslots,
-                             uint8_t* flag) {
+                             int64_t side_cap, uint8_t* flag) {
   for (int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s < nslots; s += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t b = s / kSideCap;
-    if ((uint32_t)(s - b * kSideCap) < cnt[b]) flag[ix[s]] = sflag[s];
+    const int64_t b = s / side_cap;
+    if ((uint32_t)(s - b * side_cap) < cnt[b]) flag[ix[s]] = sflag[s];
   }
 }
 cudaError_t run_slot_flags(const BucketScratch& s, int side, uint8_t* flag, cudaStream_t st) {
-  const int64_t nslots = (int64_t)s.B * kSideCap;
+  const int64_t nslots = (int64_t)s.B * s.side_cap;
   int64_t g = (nslots + 255) / 256;
   if (g > 148 * 16) g = 148 * 16;
   count_launch();
-  k_slot_flags<<<(unsigned)g, 256, 0, st>>>(s.bcnt + (side ? s.B : 0), s.ix[side], s.sflag[side], nslots, flag);
+  k_slot_flags<<<(unsigned)g, 256, 0, st>>>(s.bcnt + (side ? s.B : 0), s.ix[side], s.sflag[side], nslots, s.side_cap,
+                                            flag);
   return cudaGetLastError();
 }
 

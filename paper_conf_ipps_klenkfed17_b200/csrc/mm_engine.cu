@@ -437,8 +437,9 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
          ensure(e->scan, (size_t)scan_scratch_elems(n) * 8) == cudaSuccess;
     // bucket regions sized for the larger side (k_bucket.cu)
     const int64_t side = e->rcap > e->mcap ? e->rcap : e->mcap;
-    const PartPlan pl = part_plan_alloc(side);
-    const int64_t nbk = bucket_count(side), slots = nbk * pl.cap[pl.passes - 1];
+    const int avg = bucket_avg(semantics == MM_SEM_NOWILD_ORDERED);
+    const PartPlan pl = part_plan_alloc(side, avg);
+    const int64_t nbk = bucket_count(side, avg), slots = nbk * pl.cap[pl.passes - 1];
     for (int b = 0; ok && b < 2; b++) {
       ok = ensure(e->bh[b], (size_t)slots * 8) == cudaSuccess && ensure(e->bix[b], (size_t)slots * 4) == cudaSuccess &&
            ensure(e->bsflag[b], (size_t)slots) == cudaSuccess;
@@ -833,7 +834,7 @@ static int flat_tail(mm_engine* e, const FlatArgs& a, const BucketScratch& bs, b
                         ss.part, hs.owner, hs.tkey, e->fb_dev.p};
   static_assert(sizeof(ptrs) == sizeof(key.ptr), "TailKey pointers");
   memcpy(key.ptr, ptrs, sizeof(ptrs));
-  const int64_t vals[] = {res[0], res[1], ns[0], ns[1], (int64_t)bs.B, ordered ? 1 : 0, hs.T, 0};
+  const int64_t vals[] = {res[0], res[1], ns[0], ns[1], (int64_t)bs.B, ordered ? 1 : 0, hs.T, bs.side_cap};
   memcpy(key.val, vals, sizeof(vals));
   mm_engine::TailGraph* t = nullptr;
   for (auto& c : e->tails)

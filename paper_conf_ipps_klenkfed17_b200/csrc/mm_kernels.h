@@ -120,8 +120,8 @@ struct PartPlan {                 // partition passes for a side of n_side eleme
   int64_t cnt_total;
   int64_t scratch_slots[2];       // intermediate levels alternate between two buffers
 };
-PartPlan part_plan(int64_t n_side);
-PartPlan part_plan_alloc(int64_t n_side);  // the largest any batch up to n_side needs
+PartPlan part_plan(int64_t n_side, int avg);
+PartPlan part_plan_alloc(int64_t n_side, int avg);  // the largest any batch up to n_side needs
 struct BucketScratch {
   uint64_t* h[2];      // final bucket regions (plan.slots[last]): headers (receives, messages)
   uint32_t* ix[2];     // ... snapshot indices
@@ -134,11 +134,13 @@ struct BucketScratch {
   uint32_t* overflow;
   int64_t rres, mres;
   PartPlan plan;       // set by run_bucketed
+  int64_t side_cap;    // region slots per side and bucket (set by run_bucketed)
   const uint32_t* bcnt;  // final counts [2][B] (set by run_bucketed)
   uint32_t B;
 };
-int bucket_bits_for(int64_t n_side);
-int64_t bucket_count(int64_t n_side);
+int bucket_avg(bool ordered);  // bucket geometry: average elements per side and bucket
+int bucket_bits_for(int64_t n_side, int avg);
+int64_t bucket_count(int64_t n_side, int avg);
 cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cudaStream_t st);
 // snapshot-order matched flags of one side from the bucket slots (partly matched sides)
 cudaError_t run_slot_flags(const BucketScratch& s, int side, uint8_t* flag, cudaStream_t st);

@@ -106,41 +106,18 @@ int main() {
   float x4 = both([&](cudaStream_t s) { rd8x4<<<296, 256, 0, s>>>(hs, dd, n); },
                   [&](cudaStream_t s) { wr8<<<296, 256, 0, s>>>(hd, n); });
   printf("64 MB each way, concurrent: memcpy+memcpy %.3f ms, memcpy H2D + kernel writes %.3f ms, kernel reads + memcpy D2H %.3f ms, kernel reads + kernel writes %.3f ms\n", x1, x2, x3, x4);
-  // copy pattern of the host pipeline (no kernels) for range-weight shapes,
-  // each repeated; H2D of range k (both halves) on s1, D2H of range k on s2
-  // after it
-  const std::vector<std::vector<int>> shapes = {
-      {1, 1, 1, 1}, {1, 4, 4, 4, 2, 1}, {1, 1, 1, 1, 1, 1, 1, 1}, {1, 2, 2, 2, 1}, {1, 2, 3, 3, 2, 1}, {1, 3, 3, 3, 1}};
-  const int64_t shift_el = getenv("SHIFT") ? atoll(getenv("SHIFT")) : 0;
-  for (int rep = 0; rep < 2; rep++)
-    for (int sh = 0; sh < 3; sh++)
-    for (const auto& w : shapes) {
-      const int64_t sft = sh == 0 ? 0 : (sh == 1 ? 1024 : 37 * 1024);
-      const int C = (int)w.size();
-      int64_t wsum = 0, off[65];
-      for (int x : w) wsum += x;
-      off[0] = 0;
-      int64_t acc = 0;
-      for (int j = 0; j < C; j++) { acc += w[j]; off[j + 1] = (int64_t)(n / 2) * acc / wsum + (j + 1 < C ? sft : 0); }
-      cudaEvent_t ev[64];
-      for (int j = 0; j < C; j++) cudaEventCreateWithFlags(&ev[j], cudaEventDisableTiming);
-      float t = both([&](cudaStream_t s) {
-        for (int j = 0; j < C; j++) {
-          cudaMemcpyAsync(ds + off[j], hs + off[j], (off[j + 1] - off[j]) * 8, cudaMemcpyHostToDevice, s);
-          cudaMemcpyAsync(ds + n / 2 + off[j], hs + n / 2 + off[j], (off[j + 1] - off[j]) * 8, cudaMemcpyHostToDevice, s);
-          cudaEventRecord(ev[j], s);
-        }
-      }, [&](cudaStream_t s) {
-        for (int j = 0; j < C; j++) {
-          cudaStreamWaitEvent(s, ev[j], 0);
-          cudaMemcpyAsync(hd + off[j], dd + off[j], (off[j + 1] - off[j]) * 8, cudaMemcpyDeviceToHost, s);
-          cudaMemcpyAsync(hd + n / 2 + off[j], dd + n / 2 + off[j], (off[j + 1] - off[j]) * 8, cudaMemcpyDeviceToHost, s);
-        }
-      });
-      printf("rep %d shift %6lld el shape", rep, (long long)sft);
-      for (int x : w) printf(" %d", x);
-      printf(": %.3f ms\n", t);
+  // H2D of 64 MB in 12 copies on one stream: with and without an event
+  // record after each copy (does a record drain the copy pipeline?)
+  {
+    cudaEvent_t ev[12];
+    for (int j = 0; j < 12; j++) cudaEventCreateWithFlags(&ev[j], cudaEventDisableTiming);
+    for (int rep = 0; rep < 3; rep++) {
+      float t0 = tm([&] { for (int j = 0; j < 12; j++) cudaMemcpyAsync(ds + j * (n / 12), hs + j * (n / 12), (n / 12) * 8, cudaMemcpyHostToDevice); });
+      float t1 = tm([&] { for (int j = 0; j < 12; j++) { cudaMemcpyAsync(ds + j * (n / 12), hs + j * (n / 12), (n / 12) * 8, cudaMemcpyHostToDevice); cudaEventRecord(ev[j], 0); } });
+      float t2 = tm([&] { cudaMemcpyAsync(ds, hs, n * 8, cudaMemcpyHostToDevice); });
+      printf("H2D 64 MB: 12 copies %.3f ms, 12 copies + event records %.3f ms, 1 copy %.3f ms\n", t0, t1, t2);
     }
+  }
   printf("err %s\n", cudaGetErrorString(cudaGetLastError()));
   return 0;
 }
