@@ -635,9 +635,9 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cuda
   s.B = B;
   const int last = pl.passes - 1;
   s.bcnt = s.cnt + pl.cnt_off[last];
+  s.overflow = s.cnt + pl.cnt_total;  // cleared with the counts (one memset)
   cudaError_t err;
-  if ((err = cudaMemsetAsync(s.cnt, 0, sizeof(uint32_t) * pl.cnt_total, st)) != cudaSuccess) return err;
-  if ((err = cudaMemsetAsync(s.overflow, 0, 4, st)) != cudaSuccess) return err;
+  if ((err = cudaMemsetAsync(s.cnt, 0, sizeof(uint32_t) * (pl.cnt_total + 1), st)) != cudaSuccess) return err;
   PassArgs pa{};
   pa.snap[0] = SnapRead{a.R.q_hdr, a.R.p_hdr, s.rres};
   pa.snap[1] = SnapRead{a.M.q_hdr, a.M.p_hdr, s.mres};

@@ -415,10 +415,12 @@ __global__ void k_finalize(const int64_t* n_out_src, int64_t n_out_host, const u
 // conditional bodies -- the global fallback + compaction, or each side's
 // compaction when it is not fully matched -- so the host never reads them
 // back; a fully matched side's residual queue is emptied here.
+// Without a fallback the pair count is final here, so the gate also writes
+// the counts (the fallback body ends with its own finalize).
 __global__ void k_flat_gate(const uint32_t* over, const unsigned long long* n_matched, int64_t nr, int64_t nm,
                             cudaGraphConditionalHandle hfb, cudaGraphConditionalHandle hr,
                             cudaGraphConditionalHandle hm, int32_t* len_r, int32_t* len_m,
-                            unsigned long long* fallbacks) {
+                            unsigned long long* fallbacks, int64_t* counts, int64_t* user_counts) {
   const bool fb = *over != 0;
   const unsigned long long m = *n_matched;
   const bool pr = !fb && (int64_t)m != nr, pm = !fb && (int64_t)m != nm;
@@ -427,14 +429,23 @@ __global__ void k_flat_gate(const uint32_t* over, const unsigned long long* n_ma
   cudaGraphSetConditional(hm, pm ? 1u : 0u);
   if (!fb && !pr) *len_r = 0;
   if (!fb && !pm) *len_m = 0;
-  if (fb) *fallbacks += 1ull;
+  if (fb) {
+    *fallbacks += 1ull;
+  } else {
+    counts[0] = nr;
+    counts[1] = (int64_t)m;
+    if (user_counts) {
+      user_counts[0] = nr;
+      user_counts[1] = (int64_t)m;
+    }
+  }
 }
 cudaError_t launch_flat_gate(const uint32_t* over, const unsigned long long* n_matched, int64_t nr, int64_t nm,
                              cudaGraphConditionalHandle hfb, cudaGraphConditionalHandle hr,
                              cudaGraphConditionalHandle hm, int32_t* len_r, int32_t* len_m,
-                             unsigned long long* fallbacks, cudaStream_t st) {
+                             unsigned long long* fallbacks, int64_t* counts, int64_t* user_counts, cudaStream_t st) {
   count_launch();
-  k_flat_gate<<<1, 1, 0, st>>>(over, n_matched, nr, nm, hfb, hr, hm, len_r, len_m, fallbacks);
+  k_flat_gate<<<1, 1, 0, st>>>(over, n_matched, nr, nm, hfb, hr, hm, len_r, len_m, fallbacks, counts, user_counts);
   return cudaGetLastError();
 }
 

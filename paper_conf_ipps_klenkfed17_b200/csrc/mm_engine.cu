@@ -181,7 +181,7 @@ struct mm_engine {
   DBuf skey[2], sval[2], rid, run_start, run_rc, part;
   DBuf owner, rcnt, mcnt, tkey, tval;
   int64_t T = 0;
-  DBuf bh[2], bix[2], bsflag[2], bxh[2][2], bxix[2][2], bcnt, broff, bscan, bover;  // bucket regions (k_bucket.cu)
+  DBuf bh[2], bix[2], bsflag[2], bxh[2][2], bxix[2][2], bcnt, broff, bscan;  // bucket regions (k_bucket.cu)
   int flat_kernel = MM_FLAT_KERNEL_BUCKETED;
   long long bucket_fallbacks = 0;
   // Device-decided tail of bucketed no-wildcard batches (flat_tail): a CUDA
@@ -191,7 +191,7 @@ struct mm_engine {
   // cached by everything their launches capture (TailKey).
   struct TailKey {
     FlatArgs a;
-    const void* ptr[24];
+    const void* ptr[26];
     int64_t val[8];
   };
   struct TailGraph {
@@ -205,6 +205,7 @@ struct mm_engine {
   cudaStream_t gs = nullptr;  // capture stream
   DBuf fb_dev;                // fallbacks taken by device-decided tails
   int tail_mode = 1;          // MM_FLAT_TAIL A/B: 0 = host read-back of the overflow flag and the pair count
+  bool nm_zero = false;       // the pair counter is zero (mm_reset's kernel cleared it, no batch since)
   Timer timer;
   long long launches = 0;
   // host-buffer pipeline: H2D copies on cs, D2H copies on ds, chunk kernels on st
@@ -363,7 +364,7 @@ int mm_destroy(mm_engine* e) {
                   &e->sval[0], &e->sval[1], &e->rid, &e->run_start, &e->run_rc, &e->part,
                   &e->owner, &e->rcnt, &e->mcnt, &e->tkey, &e->tval, &e->fifo_ws,
                   &e->bh[0], &e->bh[1], &e->bix[0], &e->bix[1], &e->bsflag[0], &e->bsflag[1], &e->bcnt,
-                  &e->broff, &e->bscan, &e->bover, &e->bxh[0][0], &e->bxh[0][1], &e->bxh[1][0], &e->bxh[1][1],
+                  &e->broff, &e->bscan, &e->bxh[0][0], &e->bxh[0][1], &e->bxh[1][0], &e->bxh[1][1],
                   &e->bxix[0][0], &e->bxix[0][1], &e->bxix[1][0], &e->bxix[1][1], &e->fb_dev};
   for (DBuf* b : bufs) release(*b);
   delete e;
@@ -448,9 +449,9 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
           ok = ensure(e->bxh[x][b], (size_t)pl.scratch_slots[x] * 8) == cudaSuccess &&
                ensure(e->bxix[x][b], (size_t)pl.scratch_slots[x] * 4) == cudaSuccess;
     }
-    ok = ok && ensure(e->bcnt, (size_t)pl.cnt_total * 4) == cudaSuccess &&
+    ok = ok && ensure(e->bcnt, (size_t)(pl.cnt_total + 1) * 4) == cudaSuccess &&
          ensure(e->broff, (size_t)(nbk + 1) * 4) == cudaSuccess &&
-         ensure(e->bscan, (size_t)scan_scratch_elems(nbk) * 4) == cudaSuccess && ensure(e->bover, 4) == cudaSuccess;
+         ensure(e->bscan, (size_t)scan_scratch_elems(nbk) * 4) == cudaSuccess;
     if (ok && semantics == MM_SEM_NOWILD_ORDERED) {
       ok = ensure(e->skey[0], n * 8) == cudaSuccess && ensure(e->skey[1], n * 8) == cudaSuccess &&
            ensure(e->sval[0], n * 4) == cudaSuccess && ensure(e->sval[1], n * 4) == cudaSuccess &&
@@ -621,6 +622,7 @@ int mm_reset(mm_engine* e) {
   CK(launch_reset((int32_t*)e->rq.len[0].p, (int32_t*)e->mq.len[0].p, e->n_ep, (uint32_t*)e->err.p,
                   (unsigned long long*)e->nmatched.p, e->st));
   e->mpi_resid_empty = true;
+  e->nm_zero = true;
   Queue* qs[2] = {&e->rq, &e->mq};
   for (Queue* q : qs) {
     q->pend = Pending();
@@ -805,7 +807,7 @@ static cudaError_t add_if(cudaStream_t gs, cudaGraph_t g, cudaGraphNode_t dep, c
 // compaction} -> IF(messages partly matched) {slot flags, compaction}; a
 // fully matched side's residual queue is emptied by the gate.
 static int flat_tail(mm_engine* e, const FlatArgs& a, const BucketScratch& bs, bool ordered, const int64_t res[2],
-                     const int64_t ns[2]) {
+                     const int64_t ns[2], int64_t* user_counts) {
   Queue* qs[2] = {&e->rq, &e->mq};
   SortScratch ss;
   for (int b = 0; b < 2; b++) {
@@ -831,7 +833,7 @@ static int flat_tail(mm_engine* e, const FlatArgs& a, const BucketScratch& bs, b
                         e->rq.hdr[e->rq.cur ^ 1].p, e->rq.cookie[e->rq.cur ^ 1].p, e->rq.len[e->rq.cur ^ 1].p,
                         e->mq.hdr[e->mq.cur ^ 1].p, e->mq.cookie[e->mq.cur ^ 1].p, e->mq.len[e->mq.cur ^ 1].p,
                         e->scan.p, ss.key[0], ss.key[1], ss.val[0], ss.val[1], ss.rid, ss.run_start, ss.run_rc,
-                        ss.part, hs.owner, hs.tkey, e->fb_dev.p};
+                        ss.part, hs.owner, hs.tkey, e->fb_dev.p, e->counts_dev.p, user_counts};
   static_assert(sizeof(ptrs) == sizeof(key.ptr), "TailKey pointers");
   memcpy(key.ptr, ptrs, sizeof(ptrs));
   const int64_t vals[] = {res[0], res[1], ns[0], ns[1], (int64_t)bs.B, ordered ? 1 : 0, hs.T, bs.side_cap};
@@ -854,7 +856,7 @@ static int flat_tail(mm_engine* e, const FlatArgs& a, const BucketScratch& bs, b
       err = capture_into(e->gs, g, [&](cudaStream_t st) {
         return launch_flat_gate(bs.overflow, a.n_matched, a.nr, a.nm, h[0], h[1], h[2],
                                 (int32_t*)e->rq.len[e->rq.cur ^ 1].p, (int32_t*)e->mq.len[e->mq.cur ^ 1].p,
-                                (unsigned long long*)e->fb_dev.p, st);
+                                (unsigned long long*)e->fb_dev.p, (int64_t*)e->counts_dev.p, user_counts, st);
       });
     cudaGraphNode_t prev = nullptr;
     size_t nn = 1;
@@ -872,6 +874,8 @@ static int flat_tail(mm_engine* e, const FlatArgs& a, const BucketScratch& bs, b
         if (r == cudaSuccess) r = ordered ? run_sort_rank(a, 0ull, ~0ull, ss, st) : run_hash(a, hs, st);
         if (r == cudaSuccess) r = compact(0, a.rflag, st);
         if (r == cudaSuccess) r = compact(1, a.mflag, st);
+        if (r == cudaSuccess)
+          r = launch_finalize(nullptr, a.nr, a.n_matched, (int64_t*)e->counts_dev.p, user_counts, st);
         return r;
       });
     for (int i = 0; i < 2 && err == cudaSuccess; i++)
@@ -927,7 +931,8 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
     drc = (int64_t*)e->out_rc_stage.p;
     dmc = (int64_t*)e->out_mc_stage.p;
   }
-  CK(cudaMemsetAsync(e->nmatched.p, 0, 8, e->st));
+  if (!e->nm_zero) CK(cudaMemsetAsync(e->nmatched.p, 0, 8, e->st));
+  e->nm_zero = false;
   FlatArgs a;
   a.R = R;
   a.M = M;
@@ -954,7 +959,6 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
     bs.cnt = (uint32_t*)e->bcnt.p;
     bs.roff = (uint32_t*)e->broff.p;
     bs.scan = (uint32_t*)e->bscan.p;
-    bs.overflow = (uint32_t*)e->bover.p;
     bs.rres = info.rres;
     bs.mres = info.mres;
     e->timer.begin(e->st);
@@ -962,10 +966,8 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
     e->timer.end(e->st);
     if (e->tail_mode) {
       const int64_t res[2] = {info.rres, info.mres}, ns[2] = {nr, nm};
-      const int tr = flat_tail(e, a, bs, ordered, res, ns);
-      if (tr != MM_OK) return tr;
-      CK(launch_finalize(nullptr, nr, (const unsigned long long*)e->nmatched.p, (int64_t*)e->counts_dev.p,
-                         counts && !counts_host ? counts : nullptr, e->st));
+      const int tr = flat_tail(e, a, bs, ordered, res, ns, counts && !counts_host ? counts : nullptr);
+      if (tr != MM_OK) return tr;  // (the tail writes the counts)
       // the residual sizes are known again only if the pair count comes back
       // anyway (host outputs or host counts: the call synchronises)
       const bool back = host_out || counts_host;
@@ -981,7 +983,7 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
       }
       return dr;
     }
-    CK(cudaMemcpyAsync(&e->h_small->over, e->bover.p, 4, cudaMemcpyDeviceToHost, e->st));
+    CK(cudaMemcpyAsync(&e->h_small->over, bs.overflow, 4, cudaMemcpyDeviceToHost, e->st));
     CK(cudaMemcpyAsync(&e->h_small->matched, e->nmatched.p, 8, cudaMemcpyDeviceToHost, e->st));
     CK(cudaStreamSynchronize(e->st));
     matched_host = e->h_small->matched;

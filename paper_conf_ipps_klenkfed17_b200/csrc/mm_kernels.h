@@ -98,12 +98,13 @@ cudaError_t run_hash(const FlatArgs& a, const HashScratch& h, cudaStream_t st);
 
 // Gate of the device-decided tail of a bucketed batch (one thread): sets the
 // graph's conditional handles (fallback / partly matched receives / partly
-// matched messages), empties the residual queue of a fully matched side and
-// counts fallbacks.
+// matched messages), empties the residual queue of a fully matched side,
+// counts fallbacks and, without one, writes the counts {nr, pairs} (engine
+// and, if given, caller).
 cudaError_t launch_flat_gate(const uint32_t* over, const unsigned long long* n_matched, int64_t nr, int64_t nm,
                              cudaGraphConditionalHandle hfb, cudaGraphConditionalHandle hr,
                              cudaGraphConditionalHandle hm, int32_t* len_r, int32_t* len_m,
-                             unsigned long long* fallbacks, cudaStream_t st);
+                             unsigned long long* fallbacks, int64_t* counts, int64_t* user_counts, cudaStream_t st);
 
 // Both no-wildcard levels, hash-bucketed (k_bucket.cu): one-pass partition
 // into fixed-capacity bucket regions + one CTA per bucket.  Sets *overflow if
@@ -128,10 +129,10 @@ struct BucketScratch {
   uint8_t* sflag[2];   // ... matched byte per slot
   uint64_t* xh[2][2];  // intermediate regions [buffer][side]
   uint32_t* xix[2][2];
-  uint32_t* cnt;       // every pass's region counts (plan.cnt_total)
+  uint32_t* cnt;       // every pass's region counts (plan.cnt_total), then the overflow flag
   uint32_t* roff;      // [B + 1] output offsets of the buckets
   uint32_t* scan;      // scan scratch (scan_scratch_elems(B))
-  uint32_t* overflow;
+  uint32_t* overflow;  // = cnt + plan.cnt_total (set by run_bucketed)
   int64_t rres, mres;
   PartPlan plan;       // set by run_bucketed
   int64_t side_cap;    // region slots per side and bucket (set by run_bucketed)
