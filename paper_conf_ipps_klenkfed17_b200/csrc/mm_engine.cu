@@ -217,8 +217,14 @@ struct mm_engine {
   struct Small {
     SnapInfo info;
     unsigned long long matched;
+    unsigned long long tail_matched;  // pair count of the last device-decided tail (read back asynchronously)
     uint32_t over;
   }* h_small = nullptr;
+  // after a device-decided tail with device buffers the residual sizes are
+  // exact again (resid_host = snapshot - pairs) once ev_nm has completed:
+  // the next batch then fetches the pair count on the side stream
+  cudaEvent_t ev_nm = nullptr;
+  bool nm_pending = false;
   int pipeline = 0;          // MM_OPT_PIPELINE_CHUNKS (0 = auto)
   int host_out = MM_HOST_OUT_STAGED;  // MM_OPT_HOST_OUT
   // copies out of the caller's host input buffers still in flight: recorded
@@ -345,6 +351,7 @@ int mm_destroy(mm_engine* e) {
   for (auto& t : e->tails)
     if (t.exec) cudaGraphExecDestroy(t.exec);
   if (e->gs) cudaStreamDestroy(e->gs);
+  if (e->ev_nm) cudaEventDestroy(e->ev_nm);
   if (e->cs) cudaStreamDestroy(e->cs);
   if (e->ds) cudaStreamDestroy(e->ds);
   if (e->h_off) cudaFreeHost(e->h_off);
@@ -412,6 +419,7 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
        cudaEventCreateWithFlags(&e->ev_in_cs, cudaEventDisableTiming) == cudaSuccess;
   if (ok && semantics != MM_SEM_MPI) {
     ok = cudaStreamCreateWithFlags(&e->gs, cudaStreamNonBlocking) == cudaSuccess &&
+         cudaEventCreateWithFlags(&e->ev_nm, cudaEventDisableTiming) == cudaSuccess &&
          ensure(e->fb_dev, 8) == cudaSuccess && cudaMemset(e->fb_dev.p, 0, 8) == cudaSuccess;
     e->tail_mode = MM_FLAT_TAIL;
   }
@@ -623,6 +631,7 @@ int mm_reset(mm_engine* e) {
                   (unsigned long long*)e->nmatched.p, e->st));
   e->mpi_resid_empty = true;
   e->nm_zero = true;
+  e->nm_pending = false;
   Queue* qs[2] = {&e->rq, &e->mq};
   for (Queue* q : qs) {
     q->pend = Pending();
@@ -905,6 +914,20 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
   const bool counts_host = counts && !is_device_ptr(counts);
   const bool ordered = e->sem == MM_SEM_NOWILD_ORDERED;
   Side R = make_side(e, e->rq, e->rcap), M = make_side(e, e->mq, e->mcap);
+  // the previous device-decided tail has completed (always so when the
+  // caller synchronised since, e.g. the sharded path's count exchange): its
+  // final pair count is fetched on the side stream -- the engine stream is
+  // not waited for -- and the residual sizes are exact again
+  if (e->nm_pending && cudaEventQuery(e->ev_nm) == cudaSuccess) {
+    e->nm_pending = false;
+    CK(cudaMemcpyAsync(&e->h_small->tail_matched, e->nmatched.p, 8, cudaMemcpyDeviceToHost, e->gs));
+    CK(cudaStreamSynchronize(e->gs));
+    for (Queue* q : {&e->rq, &e->mq}) {
+      q->resid_host -= (int64_t)e->h_small->tail_matched;
+      q->resid_exact = true;
+    }
+  }
+  cudaGetLastError();  // (a not-yet-complete query is not an error)
   // exact residual sizes (and, for the sort, the varying header bits)
   const int64_t bound = e->rq.resid_host + R.p_n + e->mq.resid_host + M.p_n;
   // the varying header bits (diff) are only needed by the global sort; the
@@ -970,17 +993,22 @@ static int match_flat(mm_engine* e, int64_t* out_rc, int64_t* out_mc, int64_t ou
       if (tr != MM_OK) return tr;  // (the tail writes the counts)
       // the residual sizes are known again only if the pair count comes back
       // anyway (host outputs or host counts: the call synchronises)
+      // exact residual sizes at once if this call synchronises anyway (host
+      // outputs or host counts: the pair count comes back with them), else
+      // from the next batch on once this tail has completed (ev_nm)
       const bool back = host_out || counts_host;
-      if (back) CK(cudaMemcpyAsync(&e->h_small->matched, e->nmatched.p, 8, cudaMemcpyDeviceToHost, e->st));
+      if (back) CK(cudaMemcpyAsync(&e->h_small->tail_matched, e->nmatched.p, 8, cudaMemcpyDeviceToHost, e->st));
+      else CK(cudaEventRecord(e->ev_nm, e->st));
       const int dr = deliver(e, out_rc, out_mc, host_out, nr < out_cap ? nr : out_cap, counts, counts_host);
       Queue* qs2[2] = {&e->rq, &e->mq};
       const int64_t ns2[2] = {nr, nm};
       for (int i = 0; i < 2; i++) {
         qs2[i]->cur ^= 1;
         qs2[i]->pend = Pending();
-        qs2[i]->resid_host = back ? ns2[i] - (int64_t)e->h_small->matched : ns2[i];
+        qs2[i]->resid_host = back ? ns2[i] - (int64_t)e->h_small->tail_matched : ns2[i];
         qs2[i]->resid_exact = back;
       }
+      e->nm_pending = !back;
       return dr;
     }
     CK(cudaMemcpyAsync(&e->h_small->over, bs.overflow, 4, cudaMemcpyDeviceToHost, e->st));
@@ -1125,6 +1153,7 @@ int mm_query(mm_engine* e, int64_t* vals) {
   if (e->fb_dev.p) CK(cudaMemcpy(&fbd, e->fb_dev.p, 8, cudaMemcpyDeviceToHost));
   vals[MM_Q_FALLBACKS] = e->bucket_fallbacks + (int64_t)fbd;
   if (e->sem != MM_SEM_MPI) {
+    e->nm_pending = false;
     e->rq.resid_host = rsum;
     e->mq.resid_host = msum;
     e->rq.resid_exact = e->mq.resid_exact = true;

@@ -444,6 +444,44 @@ def test_ordered_all_same_key(flat):
 
 
 @pytest.mark.parametrize("sem", [ORD, UNO], ids=["ordered", "unordered"])
+def test_nowild_batches_back_to_back(sem):
+    """Device buffers, batches enqueued back to back with no synchronisation
+    in between (the previous tail's pair count may still be in flight when the
+    next batch is sized): per batch identical to the oracle (ordered) / valid
+    and maximal (unordered), residual depths exact at the end."""
+    import torch
+    from _util import to_dev
+    from paper_conf_ipps_klenkfed17_b200 import Engine
+    rng = np.random.default_rng(9)
+    q = synth.nowild_pairs(21, n=60000, n_src=500, n_tag=4, p_unmatched=0.3)
+    batches = split_batches(q, 5, rng)
+    eng = Engine(sem, 1, 120000, 120000)
+    outs = []
+    for (rh, rc, ro, mh, mc, mo) in batches:
+        eng.post_recvs(to_dev(rh), to_dev(rc), to_dev(ro))
+        eng.push_msgs(to_dev(mh), to_dev(mc), to_dev(mo))
+        orc = torch.full((120000,), -7, dtype=torch.int64, device="cuda")
+        omc = torch.full((120000,), -7, dtype=torch.int64, device="cuda")
+        cnt = torch.zeros(2, dtype=torch.int64, device="cuda")
+        eng.match_batch(orc, omc, cnt)
+        outs.append((orc, omc, cnt))
+    torch.cuda.synchronize()
+    g = []
+    for orc, omc, cnt in outs:
+        c = cnt.cpu().numpy()
+        g.append((orc[: c[0]].cpu().numpy(), omc[: c[0]].cpu().numpy(), c))
+    qs = eng.query()
+    eng.close()
+    if sem == ORD:
+        o, oe = oracle_batches(ORD, 1, batches)
+        assert_same_pairs(g, o)
+        rr, rm = oe.residual_depths()
+        assert qs["resid_recv"] == sum(rr) and qs["resid_msg"] == sum(rm)
+    else:
+        check_unordered_per_batch(g, batches, q.recv_hdr, q.msg_hdr)
+
+
+@pytest.mark.parametrize("sem", [ORD, UNO], ids=["ordered", "unordered"])
 @pytest.mark.parametrize("host", [False, True], ids=["dev", "host"])
 def test_bucket_fallback_between_bucketed_batches(sem, host):
     """Batch 1 overflows the buckets (one tuple repeated thousands of times:
