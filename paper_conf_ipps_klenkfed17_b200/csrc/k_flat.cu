@@ -419,14 +419,15 @@ __global__ void k_finalize(const int64_t* n_out_src, int64_t n_out_host, const u
 // the counts (the fallback body ends with its own finalize).
 __global__ void k_flat_gate(const uint32_t* over, const unsigned long long* n_matched, int64_t nr, int64_t nm,
                             cudaGraphConditionalHandle hfb, cudaGraphConditionalHandle hr,
-                            cudaGraphConditionalHandle hm, int32_t* len_r, int32_t* len_m,
-                            unsigned long long* fallbacks, int64_t* counts, int64_t* user_counts) {
+                            cudaGraphConditionalHandle hm, cudaGraphConditionalHandle hany, int32_t* len_r,
+                            int32_t* len_m, unsigned long long* fallbacks, int64_t* counts, int64_t* user_counts) {
   const bool fb = *over != 0;
   const unsigned long long m = *n_matched;
   const bool pr = !fb && (int64_t)m != nr, pm = !fb && (int64_t)m != nm;
   cudaGraphSetConditional(hfb, fb ? 1u : 0u);
   cudaGraphSetConditional(hr, pr ? 1u : 0u);
   cudaGraphSetConditional(hm, pm ? 1u : 0u);
+  cudaGraphSetConditional(hany, (fb || pr || pm) ? 1u : 0u);
   if (!fb && !pr) *len_r = 0;
   if (!fb && !pm) *len_m = 0;
   if (fb) {
@@ -442,10 +443,12 @@ __global__ void k_flat_gate(const uint32_t* over, const unsigned long long* n_ma
 }
 cudaError_t launch_flat_gate(const uint32_t* over, const unsigned long long* n_matched, int64_t nr, int64_t nm,
                              cudaGraphConditionalHandle hfb, cudaGraphConditionalHandle hr,
-                             cudaGraphConditionalHandle hm, int32_t* len_r, int32_t* len_m,
-                             unsigned long long* fallbacks, int64_t* counts, int64_t* user_counts, cudaStream_t st) {
+                             cudaGraphConditionalHandle hm, cudaGraphConditionalHandle hany, int32_t* len_r,
+                             int32_t* len_m, unsigned long long* fallbacks, int64_t* counts, int64_t* user_counts,
+                             cudaStream_t st) {
   count_launch();
-  k_flat_gate<<<1, 1, 0, st>>>(over, n_matched, nr, nm, hfb, hr, hm, len_r, len_m, fallbacks, counts, user_counts);
+  k_flat_gate<<<1, 1, 0, st>>>(over, n_matched, nr, nm, hfb, hr, hm, hany, len_r, len_m, fallbacks, counts,
+                               user_counts);
   return cudaGetLastError();
 }
 

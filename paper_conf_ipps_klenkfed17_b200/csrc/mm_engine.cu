@@ -157,6 +157,9 @@ struct Queue {
 
 }  // namespace
 
+#ifndef MM_TAIL_SIDE
+#define MM_TAIL_SIDE 1  // A/B: the tail graph launched on the side stream
+#endif
 #ifndef MM_FLAT_TAIL
 #define MM_FLAT_TAIL 1  // device-decided tail of bucketed no-wildcard batches (0: host read-back)
 #endif
@@ -225,6 +228,7 @@ struct mm_engine {
   // the next batch then fetches the pair count on the side stream
   cudaEvent_t ev_nm = nullptr;
   bool nm_pending = false;
+  cudaEvent_t ev_tail[2] = {nullptr, nullptr};  // orders the tail graph's side-stream launch
   int pipeline = 0;          // MM_OPT_PIPELINE_CHUNKS (0 = auto)
   int host_out = MM_HOST_OUT_STAGED;  // MM_OPT_HOST_OUT
   // copies out of the caller's host input buffers still in flight: recorded
@@ -352,6 +356,8 @@ int mm_destroy(mm_engine* e) {
     if (t.exec) cudaGraphExecDestroy(t.exec);
   if (e->gs) cudaStreamDestroy(e->gs);
   if (e->ev_nm) cudaEventDestroy(e->ev_nm);
+  for (cudaEvent_t ev : e->ev_tail)
+    if (ev) cudaEventDestroy(ev);
   if (e->cs) cudaStreamDestroy(e->cs);
   if (e->ds) cudaStreamDestroy(e->ds);
   if (e->h_off) cudaFreeHost(e->h_off);
@@ -420,6 +426,8 @@ int mm_create(mm_engine** out, int32_t semantics, int32_t n_endpoints, int64_t r
   if (ok && semantics != MM_SEM_MPI) {
     ok = cudaStreamCreateWithFlags(&e->gs, cudaStreamNonBlocking) == cudaSuccess &&
          cudaEventCreateWithFlags(&e->ev_nm, cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&e->ev_tail[0], cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&e->ev_tail[1], cudaEventDisableTiming) == cudaSuccess &&
          ensure(e->fb_dev, 8) == cudaSuccess && cudaMemset(e->fb_dev.p, 0, 8) == cudaSuccess;
     e->tail_mode = MM_FLAT_TAIL;
   }
@@ -802,9 +810,22 @@ static cudaError_t add_if(cudaStream_t gs, cudaGraph_t g, cudaGraphNode_t dep, c
   p.conditional.handle = h;
   p.conditional.type = cudaGraphCondTypeIf;
   p.conditional.size = 1;
-  cudaError_t err = cudaGraphAddNode(node, g, &dep, 1, &p);
+  cudaError_t err = cudaGraphAddNode(node, g, dep ? &dep : nullptr, dep ? 1 : 0, &p);
   if (err != cudaSuccess) return err;
   return capture_into(gs, p.conditional.phGraph_out[0], f);
+}
+
+// Append an IF node (after dep) and return its (empty) body graph.
+static cudaError_t add_if_body(cudaGraph_t g, cudaGraphNode_t dep, cudaGraphConditionalHandle h, cudaGraphNode_t* node,
+                               cudaGraph_t* body) {
+  cudaGraphNodeParams p = {};
+  p.type = cudaGraphNodeTypeConditional;
+  p.conditional.handle = h;
+  p.conditional.type = cudaGraphCondTypeIf;
+  p.conditional.size = 1;
+  cudaError_t err = cudaGraphAddNode(node, g, &dep, 1, &p);
+  if (err == cudaSuccess) *body = p.conditional.phGraph_out[0];
+  return err;
 }
 
 }  // extern "C++"
@@ -858,12 +879,14 @@ static int flat_tail(mm_engine* e, const FlatArgs& a, const BucketScratch& bs, b
     t->exec = nullptr;
     cudaGraph_t g;
     CK(cudaGraphCreate(&g, 0));
-    cudaGraphConditionalHandle h[3];
+    // h[3]: anything to do at all -- the common all-matched batch evaluates
+    // one conditional node (each costs ~9 us of GPU time even when false)
+    cudaGraphConditionalHandle h[4];
     cudaError_t err = cudaSuccess;
-    for (int i = 0; i < 3 && err == cudaSuccess; i++) err = cudaGraphConditionalHandleCreate(&h[i], g, 0, cudaGraphCondAssignDefault);
+    for (int i = 0; i < 4 && err == cudaSuccess; i++) err = cudaGraphConditionalHandleCreate(&h[i], g, 0, cudaGraphCondAssignDefault);
     if (err == cudaSuccess)
       err = capture_into(e->gs, g, [&](cudaStream_t st) {
-        return launch_flat_gate(bs.overflow, a.n_matched, a.nr, a.nm, h[0], h[1], h[2],
+        return launch_flat_gate(bs.overflow, a.n_matched, a.nr, a.nm, h[0], h[1], h[2], h[3],
                                 (int32_t*)e->rq.len[e->rq.cur ^ 1].p, (int32_t*)e->mq.len[e->mq.cur ^ 1].p,
                                 (unsigned long long*)e->fb_dev.p, (int64_t*)e->counts_dev.p, user_counts, st);
       });
@@ -876,9 +899,11 @@ static int flat_tail(mm_engine* e, const FlatArgs& a, const BucketScratch& bs, b
       return run_compact(i ? a.M : a.R, res[i], ns[i], flags, (uint64_t*)q.hdr[nb].p, (int64_t*)q.cookie[nb].p,
                          (int32_t*)q.len[nb].p, (uint32_t*)e->scan.p, st);
     };
-    cudaGraphNode_t n0, n1, n2;
+    cudaGraphNode_t nany, n0, n1, n2;
+    cudaGraph_t body = nullptr;
+    if (err == cudaSuccess) err = add_if_body(g, prev, h[3], &nany, &body);
     if (err == cudaSuccess)
-      err = add_if(e->gs, g, prev, h[0], &n0, [&](cudaStream_t st) {
+      err = add_if(e->gs, body, nullptr, h[0], &n0, [&](cudaStream_t st) {
         cudaError_t r = cudaMemsetAsync(a.n_matched, 0, 8, st);
         if (r == cudaSuccess) r = ordered ? run_sort_rank(a, 0ull, ~0ull, ss, st) : run_hash(a, hs, st);
         if (r == cudaSuccess) r = compact(0, a.rflag, st);
@@ -888,7 +913,7 @@ static int flat_tail(mm_engine* e, const FlatArgs& a, const BucketScratch& bs, b
         return r;
       });
     for (int i = 0; i < 2 && err == cudaSuccess; i++)
-      err = add_if(e->gs, g, i ? n1 : n0, h[1 + i], i ? &n2 : &n1, [&](cudaStream_t st) {
+      err = add_if(e->gs, body, i ? n1 : n0, h[1 + i], i ? &n2 : &n1, [&](cudaStream_t st) {
         uint8_t* fl = i ? a.mflag : a.rflag;
         cudaError_t r = run_slot_flags(bs, i, fl, st);
         if (r == cudaSuccess) r = compact(i, fl, st);
@@ -905,7 +930,18 @@ static int flat_tail(mm_engine* e, const FlatArgs& a, const BucketScratch& bs, b
   }
   t->stamp = ++e->tail_clock;
   count_launch();  // the gate; the bodies run only when it says so
+#if MM_TAIL_SIDE
+  // launched on the side stream, ordered by events: a graph launched into the
+  // legacy default stream returned only once it had run (a ~27 us gap per
+  // step before the next batch's launches)
+  CK(cudaEventRecord(e->ev_tail[0], e->st));
+  CK(cudaStreamWaitEvent(e->gs, e->ev_tail[0], 0));
+  CK(cudaGraphLaunch(t->exec, e->gs));
+  CK(cudaEventRecord(e->ev_tail[1], e->gs));
+  CK(cudaStreamWaitEvent(e->st, e->ev_tail[1], 0));
+#else
   CK(cudaGraphLaunch(t->exec, e->st));
+#endif
   return MM_OK;
 }
 

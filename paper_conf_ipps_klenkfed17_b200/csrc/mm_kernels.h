@@ -103,8 +103,9 @@ cudaError_t run_hash(const FlatArgs& a, const HashScratch& h, cudaStream_t st);
 // and, if given, caller).
 cudaError_t launch_flat_gate(const uint32_t* over, const unsigned long long* n_matched, int64_t nr, int64_t nm,
                              cudaGraphConditionalHandle hfb, cudaGraphConditionalHandle hr,
-                             cudaGraphConditionalHandle hm, int32_t* len_r, int32_t* len_m,
-                             unsigned long long* fallbacks, int64_t* counts, int64_t* user_counts, cudaStream_t st);
+                             cudaGraphConditionalHandle hm, cudaGraphConditionalHandle hany, int32_t* len_r,
+                             int32_t* len_m, unsigned long long* fallbacks, int64_t* counts, int64_t* user_counts,
+                             cudaStream_t st);
 
 // Both no-wildcard levels, hash-bucketed (k_bucket.cu): one-pass partition
 // into fixed-capacity bucket regions + one CTA per bucket.  Sets *overflow if
