@@ -77,6 +77,9 @@ int64_t bucket_count(int64_t n_side, int avg) { return (int64_t)1 << bucket_bits
 #ifndef MM_PASS_ITEMS
 #define MM_PASS_ITEMS 8
 #endif
+#ifndef MM_PASS_VEC
+#define MM_PASS_VEC 1  // A/B: later passes load element pairs with vector loads
+#endif
 #ifndef MM_PASS_MINB
 #define MM_PASS_MINB 2
 #endif
@@ -188,23 +191,51 @@ __global__ void __launch_bounds__(kPassThreads, MM_PASS_MINB) k_part_pass(PassAr
   uint64_t h[kPassItems];
   uint32_t ix[kPassItems], key[kPassItems], rank[kPassItems];
   const int64_t rbase = FIRST ? 0 : (int64_t)parent * a.icap;
+  // element of item u: later passes read pairs of consecutive elements with
+  // one 16-byte (headers) and one 8-byte (indices) load (MM_PASS_VEC); the
+  // order inside a digit run is free, so any mapping of elements to threads
+  // is valid
+  auto elem = [&](int u) -> int64_t {
+    if (!FIRST && MM_PASS_VEC) return t0 + (int64_t)(u >> 1) * (2 * kPassThreads) + 2 * tid + (u & 1);
+    return t0 + (int64_t)u * kPassThreads + tid;
+  };
+  if (!FIRST && MM_PASS_VEC) {
+    const uint64_t* ih = (sd ? a.ih[1] : a.ih[0]) + rbase;
+    const uint32_t* iix = (sd ? a.iix[1] : a.iix[0]) + rbase;
 #pragma unroll
-  for (int u = 0; u < kPassItems; u++) {  // every load in flight first
-    const int64_t k = t0 + u * kPassThreads + tid;
-    if (k < t1) {
-      if (FIRST) {
-        const bool m = k >= a.n0;
-        ix[u] = (uint32_t)(m ? k - a.n0 : k);
-        h[u] = m ? a.snap[1].hdr(ix[u]) : a.snap[0].hdr(ix[u]);
-      } else {
-        h[u] = (sd ? a.ih[1] : a.ih[0])[rbase + k];
-        ix[u] = (sd ? a.iix[1] : a.iix[0])[rbase + k];
+    for (int v = 0; v < kPassItems / 2; v++) {  // every load in flight first
+      const int64_t k = elem(2 * v);
+      if (k + 1 < t1) {
+        const ulonglong2 hh = *reinterpret_cast<const ulonglong2*>(ih + k);
+        const uint2 xx = *reinterpret_cast<const uint2*>(iix + k);
+        h[2 * v] = hh.x;
+        h[2 * v + 1] = hh.y;
+        ix[2 * v] = xx.x;
+        ix[2 * v + 1] = xx.y;
+      } else if (k < t1) {
+        h[2 * v] = ih[k];
+        ix[2 * v] = iix[k];
+      }
+    }
+  } else {
+#pragma unroll
+    for (int u = 0; u < kPassItems; u++) {  // every load in flight first
+      const int64_t k = elem(u);
+      if (k < t1) {
+        if (FIRST) {
+          const bool m = k >= a.n0;
+          ix[u] = (uint32_t)(m ? k - a.n0 : k);
+          h[u] = m ? a.snap[1].hdr(ix[u]) : a.snap[0].hdr(ix[u]);
+        } else {
+          h[u] = (sd ? a.ih[1] : a.ih[0])[rbase + k];
+          ix[u] = (sd ? a.iix[1] : a.iix[0])[rbase + k];
+        }
       }
     }
   }
 #pragma unroll
   for (int u = 0; u < kPassItems; u++) {
-    const int64_t k = t0 + u * kPassThreads + tid;
+    const int64_t k = elem(u);
     if (k < t1) {
       const uint32_t d = (bucket_of(h[u], a.nb) >> a.shift) & (F - 1);
       key[u] = FIRST ? (k >= a.n0 ? F + d : d) : d;
@@ -242,7 +273,7 @@ __global__ void __launch_bounds__(kPassThreads, MM_PASS_MINB) k_part_pass(PassAr
   __syncthreads();
 #pragma unroll
   for (int u = 0; u < kPassItems; u++) {
-    const int64_t k = t0 + u * kPassThreads + tid;
+    const int64_t k = elem(u);
     if (k < t1) {
       const uint32_t pos = sm.lstart[key[u]] + rank[u];
       sm.h[pos] = h[u];
