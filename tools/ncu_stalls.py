@@ -16,7 +16,7 @@ fname, hdr = "?", None
 lines = collections.defaultdict(lambda: collections.Counter())
 text = {}
 for r in rows:
-    if r and r[0] == "File Name":
+    if r and r[0] in ("File Name", "File Path"):
         fname = os.path.basename(r[1])
         continue
     if r and r[0] == "Line No":
