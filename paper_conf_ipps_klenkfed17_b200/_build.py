@@ -48,6 +48,7 @@ def build_library(force=False, verbose=False, variant=""):
     extra = ["-DMM_PHASE_TIMING"] if variant == "timing" else []
     if variant and variant != "timing":  # A/B builds: -D flags from MM_AB_DEFINES (profiling aid)
         extra = ["-D" + d for d in os.environ.get("MM_AB_DEFINES", "").split()]
+        extra += os.environ.get("MM_AB_FLAGS", "").split()  # raw nvcc flags of an A/B build
     cmd = [nvcc, *NVCC_FLAGS, *extra, "-Xptxas", "-v", "-o", tmp, *sources()]
     res = subprocess.run(cmd, capture_output=True, text=True)
     with open(os.path.join(LIBDIR, "ptxas%s.log" % ("_" + variant if variant else "")), "w") as f:
