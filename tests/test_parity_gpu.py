@@ -571,6 +571,31 @@ def check_min(q):
     return sum(per_key_min(q.recv_hdr, q.msg_hdr).values())
 
 
+def test_unordered_deep_tuple_takes_the_fallback():
+    """NOWILD_UNORDERED, stack kernel (k_bucket_pop): a tuple with hundreds
+    of receives in one bucket would walk its message stack too far -- the
+    bucket flags the batch and the global hash fallback matches it: valid,
+    maximal per tuple, one fallback; a tuple of 40 stays on chip."""
+    rng = np.random.default_rng(12)
+    for deep, want in [(300, 1), (40, 0)]:
+        n = 20000
+        src = rng.integers(0, 1 << 20, n)
+        tag = rng.integers(0, 64, n)
+        hot = rng.choice(n, deep, replace=False)
+        src[hot] = 9
+        tag[hot] = 4
+        rh = synth.pack(src, tag)
+        mh = rh[rng.permutation(n)]
+        b = [(rh, None, np.array([0, n]), mh, None, np.array([0, n]))]
+        g, qs = gpu_batches(UNO, 1, n, n, b, flat_kernel=0)
+        grc, gmc, cnt = g[0]
+        assert np.array_equal(np.sort(grc), np.arange(n))
+        m = gmc >= 0
+        assert np.array_equal(rh[grc[m]], mh[gmc[m]]) and len(np.unique(gmc[m])) == int(m.sum())
+        assert int(m.sum()) == n  # every message expected
+        assert qs["fallbacks"] == want
+
+
 @pytest.mark.parametrize("seed", range(3))
 @pytest.mark.parametrize("host", [False, True], ids=["dev", "host"])
 @FLAT
