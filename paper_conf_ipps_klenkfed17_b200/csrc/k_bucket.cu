@@ -48,7 +48,10 @@ struct SnapRead {
 // geometry is per level (bucket_avg): NOWILD_ORDERED 256 elements per side
 // with 128-thread CTAs, six per SM; NOWILD_UNORDERED 512 with 256-thread
 // CTAs, three per SM (A/B).
-int bucket_avg(bool ordered) { return ordered ? 256 : 512; }
+#ifndef MM_UNORD_AVG
+#define MM_UNORD_AVG 512  // A/B: NOWILD_UNORDERED bucket geometry (512: 256 threads x 3 CTAs, 256: 128 x 6)
+#endif
+int bucket_avg(bool ordered) { return ordered ? 256 : MM_UNORD_AVG; }
 
 int bucket_bits_for(int64_t n_side, int avg) {
   int nb = 1;
@@ -881,11 +884,12 @@ cudaError_t run_bucketed(const FlatArgs& a, bool ordered, BucketScratch& s, cuda
   if (ordered) return launch_bucket_match<true, 256, 128, 6>(ma, B, st);
 #if MM_UNORD_POP
   {
-    constexpr auto kern = k_bucket_pop<512, 256, 3>;
-    const size_t smem = sizeof(PopSmem<2048, 4096, 256>);
+    constexpr int kA = MM_UNORD_AVG, kT = kA == 512 ? 256 : 128, kB = kA == 512 ? 3 : 6;
+    constexpr auto kern = k_bucket_pop<kA, kT, kB>;
+    const size_t smem = sizeof(PopSmem<4 * kA, 8 * kA, kT>);
     if ((err = ensure_dyn_smem<kern>(smem)) != cudaSuccess) return err;
     count_launch();
-    kern<<<persistent_grid<kern>(256, smem, B), 256, smem, st>>>(ma);
+    kern<<<persistent_grid<kern>(kT, smem, B), kT, smem, st>>>(ma);
     return cudaGetLastError();
   }
 #endif
