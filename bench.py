@@ -61,9 +61,12 @@ REGION_KERNELS = {
     "mpi": "k_mpi_fifo",
     "mpi_cookies": "k_mpi_fifo",
     "mpi_matrix": "k_mpi_matrix",
-    "ordered": "k_part_hist + k_scan_* + k_part_scatter (both sides, 2 passes) + k_bucket_bounds + k_bucket_pair",
-    "unordered": "k_part_hist + k_scan_* + k_part_scatter (both sides, 2 passes) + k_bucket_bounds + k_bucket_pop",
-    "unordered_256m": "k_part_hist + k_scan_* + k_part_scatter (both sides) + k_bucket_bounds + k_bucket_pop",
+    "ordered": "k_part_pass x2 (MSD partition, both sides) + k_tile_reduce/k_scan_single/k_tile_downsweep "
+               "(bucket offsets) + k_bucket_match<ordered>",
+    "unordered": "k_part_pass x2 (MSD partition, both sides) + k_tile_reduce/k_scan_single/k_tile_downsweep "
+                 "(bucket offsets) + k_bucket_pop",
+    "unordered_256m": "k_part_pass x2 (MSD partition, both sides) + k_tile_reduce/k_scan_single/k_tile_downsweep "
+                      "(bucket offsets) + k_bucket_pop",
     "mpi_worst": "k_mpi_fifo (deep-endpoint instantiation: one cluster of 8 512-thread CTAs)",
 }
 # PAPER.md's own rates (GTX1080 unless stated; other hardware: context, not target)
