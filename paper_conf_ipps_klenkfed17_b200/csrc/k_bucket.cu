@@ -639,21 +639,24 @@ __global__ void __launch_bounds__(NT, MINB) k_bucket_match(MatchArgs ma) {
 // (atomicExch on the slot word); C every receive draws a ticket p from the
 // same word (atomicAdd of 1 << 16: the old word also holds the stack head)
 // and takes the stack's p-th message, if any (a walk of p links -- groups
-// are a few elements; p >= kPopWalk flags the bucket for the global
-// fallback); D the messages' matched flags are written coalesced.
+// are a few elements; a tuple with kPopWalk or more receives has its stack
+// laid out flat once and its later receives index it: no run-length limit);
+// D the messages' matched flags are written coalesced.
 // Receives are reported in bucket order (any order is allowed, mm.h).
 constexpr uint32_t kPopWalk = 64;
 
 template <int K, int H, int NT>
 struct PopSmem {
-  uint64_t hdr[K];
+  uint64_t hdr[K];    // A..B; then (as uint16) deep tuples' stacks laid out flat
   uint32_t idx[K];
   uint32_t table[H];  // (fingerprint << 16) | representative element
   uint32_t hw[H];     // (receive tickets << 16) | message stack head
-  uint16_t nxt[K];    // message -> next message of its tuple's stack
+  uint16_t nxt[K];    // message -> next message of its tuple's stack; deep receive -> its ticket
   uint16_t slot[K];   // receive -> its tuple's slot
   uint32_t mbits[K / 32];
+  uint32_t dbits[K / 32];  // deep receives (ticket >= kPopWalk)
   uint32_t nmatch;
+  uint32_t deep, ftop;
 };
 
 template <int AVG, int NT, int MINB>
@@ -724,8 +727,15 @@ __global__ void __launch_bounds__(NT, MINB) k_bucket_pop(MatchArgs ma) {
       reinterpret_cast<uint4*>(sm.table)[x] = make_uint4(~0u, ~0u, ~0u, ~0u);
       reinterpret_cast<uint4*>(sm.hw)[x] = make_uint4(0xFFFFu, 0xFFFFu, 0xFFFFu, 0xFFFFu);
     }
-    for (uint32_t x = tid; x < kK / 32; x += NT) sm.mbits[x] = 0u;
-    if (tid == 0) sm.nmatch = 0;
+    for (uint32_t x = tid; x < kK / 32; x += NT) {
+      sm.mbits[x] = 0u;
+      sm.dbits[x] = 0u;
+    }
+    if (tid == 0) {
+      sm.nmatch = 0;
+      sm.deep = 0;
+      sm.ftop = 0;
+    }
     xnr = ynr;
     xnm = ynm;
     fetch(b + G, xnr, xnm);
@@ -754,18 +764,7 @@ __global__ void __launch_bounds__(NT, MINB) k_bucket_pop(MatchArgs ma) {
     const int64_t obase = ma.roff[b];
     const int64_t sbase = (int64_t)b * kSideCap;
     uint32_t nmatch = 0;
-    bool deep = false;
-    for (uint32_t r = tid; r < nr; r += NT) {
-      const uint32_t old = atomicAdd(&sm.hw[sm.slot[r]], 0x10000u);
-      uint32_t p = old >> 16, m = old & 0xFFFFu;
-      if (p >= kPopWalk) {
-        deep = true;
-        m = 0xFFFFu;
-      }
-      while (p > 0 && m != 0xFFFFu) {
-        m = sm.nxt[m];
-        p--;
-      }
+    auto emit = [&](uint32_t r, uint32_t m) {
       int64_t mc = MM_NO_MATCH;
       if (m != 0xFFFFu) {
         mc = a.M.cookie(0, sm.idx[m], mres, mpb);
@@ -775,11 +774,48 @@ __global__ void __launch_bounds__(NT, MINB) k_bucket_pop(MatchArgs ma) {
       a.out_rc[obase + r] = a.R.cookie(0, sm.idx[r], rres, rpb);
       a.out_mc[obase + r] = mc;
       ma.sflag[0][sbase + r] = m != 0xFFFFu;
+    };
+    for (uint32_t r = tid; r < nr; r += NT) {
+      const uint32_t old = atomicAdd(&sm.hw[sm.slot[r]], 0x10000u);
+      uint32_t p = old >> 16, m = old & 0xFFFFu;
+      if (p >= kPopWalk) {  // a deep tuple: resolved below from its flattened stack
+        sm.nxt[r] = (uint16_t)p;
+        atomicOr(&sm.dbits[r >> 5], 1u << (r & 31u));
+        sm.deep = 1u;
+        continue;
+      }
+      while (p > 0 && m != 0xFFFFu) {
+        m = sm.nxt[m];
+        p--;
+      }
+      emit(r, m);
     }
-    if (deep) atomicOr(ma.overflow, 1u);  // a tuple repeated too often for the walk: global fallback
     for (int o = 16; o; o >>= 1) nmatch += __shfl_xor_sync(kFull, nmatch, o);
     if (lane == 0 && nmatch) atomicAdd(&sm.nmatch, nmatch);
+    nmatch = 0;
     __syncthreads();
+    if (sm.deep) {  // (uniform) tuples with >= kPopWalk receives: no run-length limit
+      uint16_t* flat = reinterpret_cast<uint16_t*>(sm.hdr);  // the headers are dead after B
+      // the receive holding ticket kPopWalk flattens its tuple's message stack
+      // once; the table entry (dead after B) keeps the flat array's base | length
+      for (uint32_t r = tid; r < nr; r += NT)
+        if (((sm.dbits[r >> 5] >> (r & 31u)) & 1u) && sm.nxt[r] == kPopWalk) {
+          uint32_t len = 0;
+          for (uint32_t x = sm.hw[sm.slot[r]] & 0xFFFFu; x != 0xFFFFu; x = sm.nxt[x]) len++;
+          const uint32_t base = atomicAdd(&sm.ftop, len);
+          uint32_t q = base;
+          for (uint32_t x = sm.hw[sm.slot[r]] & 0xFFFFu; x != 0xFFFFu; x = sm.nxt[x]) flat[q++] = (uint16_t)x;
+          sm.table[sm.slot[r]] = base | (len << 16);
+        }
+      __syncthreads();
+      for (uint32_t r = tid; r < nr; r += NT)
+        if ((sm.dbits[r >> 5] >> (r & 31u)) & 1u) {
+          const uint32_t t = sm.table[sm.slot[r]], p = sm.nxt[r];
+          emit(r, p < (t >> 16) ? (uint32_t)flat[(t & 0xFFFFu) + p] : 0xFFFFu);
+        }
+      if (nmatch) atomicAdd(&sm.nmatch, nmatch);
+      __syncthreads();
+    }
     // D: the messages' matched flags
     for (uint32_t j = tid; j < nm; j += NT) ma.sflag[1][sbase + j] = (sm.mbits[j >> 5] >> (j & 31u)) & 1u;
     if (tid == 0 && sm.nmatch) atomicAdd(a.n_matched, (unsigned long long)sm.nmatch);
