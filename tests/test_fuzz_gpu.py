@@ -13,7 +13,7 @@ import pytest
 
 import oracle
 import synth
-from _util import check_unordered, gpu_batches, oracle_batches, single_batch, split_batches
+from _util import check_unordered, check_unordered_per_batch, gpu_batches, oracle_batches, single_batch, split_batches
 from test_parity_gpu import assert_exact, assert_same_pairs
 
 pytestmark = pytest.mark.gpu
@@ -84,7 +84,8 @@ def test_fuzz_ordered(seed):
     rng = np.random.default_rng(seed)
     batches = split_batches(q, nb, rng) if nb > 1 else single_batch(q)
     n = max(1, cfg["n"])
-    g, qs = gpu_batches(ORD, 1, n, n, batches, flat_kernel=flat)
+    host = [False, True, "pinned"][seed % 3]  # device buffers: device-decided tails, deferred residual sizes
+    g, qs = gpu_batches(ORD, 1, n, n, batches, flat_kernel=flat, host=host)
     o, _ = oracle_batches(ORD, 1, batches)
     assert_same_pairs(g, o)
     assert qs["error"] == 0
@@ -104,3 +105,19 @@ def test_fuzz_unordered(seed):
     keys, counts = np.unique(q.recv_hdr[orc[om]], return_counts=True)
     check_unordered(q.recv_hdr, q.msg_hdr, grc, gmc, dict(zip(keys.tolist(), counts.tolist())))
     assert int(cnt[1]) == int(om.sum()) and qs["error"] == 0
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_fuzz_unordered_multibatch(seed):
+    """NOWILD_UNORDERED over 2-3 batches with residual queues (the stack
+    kernel, the device-decided tail and its deferred residual sizes, the
+    fallback for heavily repeated tuples), per batch: valid and maximal."""
+    cfg, flat, nb = flat_config(seed + 500)
+    q = synth.nowild_pairs(seed + 500, **cfg)
+    rng = np.random.default_rng(seed)
+    batches = split_batches(q, max(2, nb), rng)
+    n = max(1, cfg["n"])
+    host = [False, True, "pinned"][seed % 3]
+    g, qs = gpu_batches(UNO, 1, n, n, batches, flat_kernel=flat, host=host)
+    check_unordered_per_batch(g, batches, q.recv_hdr, q.msg_hdr)
+    assert qs["error"] == 0
